@@ -1,0 +1,356 @@
+#!/usr/bin/env python3
+"""Benchmark: single-source SSSP GTEPS on a B200 (BASELINE.json metric).
+
+A "step" is one whole bucket-aware asynchronous Delta-stepping SSSP (all
+SURVEY §8(a) rows a5-a7: init, phase 1, phases 2&3) from one seeded source on
+the resident, PRO-reordered graph. Default workload: C4 = Kronecker scale-24
+edgefactor-16, u32 weights U{1..100}, Delta=32 (the north star's ">= 50% of
+HBM on scale-24 RMAT" config). GTEPS = m / time with m = EF * 2^SCALE input
+edges.
+
+Multi-GPU (torchrun): the graph is replicated, the 64 sources are sharded
+round-robin (sources[rank::N]), each rank runs K steps; value = N*K*m / max
+rank time ("scaling": "weak"). `--impl reference` times the CPU oracle
+(plain Dijkstra, oracle/) on a bounded sample of the same workload.
+
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PAPER_V100 = {"C3": 16.78, "C4": 20.16}  # GTEPS, PAPER Fig. 11, context only
+METRIC = "SSSP GTEPS (m/time) at 1 GPU; multi-source GTEPS at 1/2/4/8 B200; HBM GB/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=64)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C4", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--delta", type=float, default=None)
+    ap.add_argument("--no-reorder", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--sources", type=int, default=64)
+    ap.add_argument("--ctas-per-sm", type=int, default=0)
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/cpu/e2e)")
+    return ap.parse_args()
+
+
+def workload_desc(name, cfg, delta, reorder):
+    import gen
+
+    c = dict(gen.CONFIGS[name])
+    if c["kind"] == "kron":
+        d = (f"{name}: Kronecker scale-{c['scale']} edgefactor-{c['edgefactor']} (Graph500 A=.57 B=.19 C=.19 "
+             f"D=.05, scrambled, symmetrised), {c['weights']} weights, delta={delta}, reorder={'on' if reorder else 'off'}")
+    else:
+        d = (f"{name}: road-like grid {c['W']}x{c['H']} (horizontal + p={c['p']} vertical), {c['weights']} "
+             f"weights, delta={delta}, reorder={'on' if reorder else 'off'}")
+    return d, c
+
+
+class ClockSampler:
+    """NVML samples of SM clock + throttle reasons during the timed region."""
+
+    REASONS = {
+        0x0000000000000004: "sw_power_cap",
+        0x0000000000000008: "hw_slowdown",
+        0x0000000000000020: "sw_thermal_slowdown",
+        0x0000000000000040: "hw_thermal_slowdown",
+        0x0000000000000080: "hw_power_brake_slowdown",
+        0x0000000000000002: "applications_clocks_setting",
+    }
+
+    def __init__(self, dev_index):
+        self.ok = False
+        self.samples = []
+        self.reasons = set()
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.max_mhz = None
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def algorithmic_bytes(g, dist_bits, inf):
+    """SURVEY §8(d) B_alg per SSSP: 8*A_r (arc stream) + 48*V_r (row pair, dist,
+    queue push/pop, settle list, atomic) + 12*V (init + output)."""
+    reach = dist_bits != inf
+    deg = np.diff(g.row)
+    A_r = int(deg[reach].sum())
+    V_r = int(reach.sum())
+    return 8 * A_r + 48 * V_r + 12 * g.V, A_r, V_r
+
+
+def load_traffic(config):
+    """ncu dram bytes per launch of the persistent kernel, from the committed summary."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(config, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def measured_peak():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def cpu_baseline(g, sources, budget_s=30.0):
+    """The oracle as it stands (single-threaded Dijkstra) on a bounded sample."""
+    import oracle
+
+    t0 = time.perf_counter()
+    n = 0
+    for s in sources:
+        oracle.dijkstra(g.row, g.col, g.w, int(s))
+        n += 1
+        if time.perf_counter() - t0 > budget_s * 0.5:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": round(n * g.m / dt / 1e9, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"{n} source(s) of the full {g.name} graph, single-threaded binary-heap Dijkstra "
+                      f"({dt:.1f} s)"}
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    import gen
+
+    cfg = gen.CONFIGS[args.config]
+    delta = args.delta if args.delta is not None else cfg["delta"]
+    reorder = not args.no_reorder
+    desc, c = workload_desc(args.config, cfg, delta, reorder)
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        g = gen.make_config(args.config)
+        srcs = gen.sample_sources(g, args.sources, seed=7)
+        import oracle
+
+        steps = []
+        for k in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            oracle.dijkstra(g.row, g.col, g.w, int(srcs[k % len(srcs)]))
+            dt = time.perf_counter() - t0
+            if k >= args.warmup:
+                steps.append(dt)
+            if sum(steps) > 150:  # bounded: keep the reference arm within minutes
+                break
+        t = sum(steps)
+        val = len(steps) * g.m / t / 1e9
+        line = {"impl": "reference", "metric": METRIC, "value": round(val, 6), "unit": "GTEPS", "n_gpus": args.gpus,
+                "steps": len(steps), "warmup": args.warmup, "ms_per_step": round(1e3 * t / len(steps), 3),
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": cfg["weights"],
+                "data": "synthetic",
+                "config": {"workload": desc, "parallelism": "cpu oracle, rank 0 only"},
+                "cpu_baseline": {"value": round(val, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                                 "sample": f"{len(steps)} source(s) of the full graph, single-threaded Dijkstra"},
+                "e2e": {"value": round(val, 6), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+
+    if world > 1:
+        import torch.distributed as dist
+
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = local if world > 1 else 0
+    torch.cuda.set_device(dev)
+    import paper_conf_icppw_zhangczsdhay23_b200 as sssp
+
+    t_gen = time.perf_counter()
+    g = gen.make_config(args.config)
+    t_gen = time.perf_counter() - t_gen
+    sources = gen.sample_sources(g, args.sources, seed=7)
+    mine = sources[rank::world]
+    stream = torch.cuda.Stream(device=dev)
+    G = sssp.Graph(g.row, g.col, g.w, device=dev, stream=stream)
+    if args.ctas_per_sm:
+        G.set_param(sssp.SSSP_PARAM_CTAS_PER_SM, args.ctas_per_sm)
+    reorder_ms = None
+    if reorder:
+        G.reorder()
+        torch.cuda.synchronize(dev)
+        reorder_ms = G.stats()["reorder_ms"]
+    inf = 0x7F800000 if g.wtype == "f32" else 0xFFFFFFFF
+
+    def step(k):
+        G.run(int(mine[k % len(mine)]), delta)
+
+    for k in range(args.warmup):
+        step(k)
+    stream.synchronize()
+    G.kernel_time(reset=True)
+
+    # ---------------- timed region (device events on the library's stream)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize(dev)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(dev)
+    with sampler if not args.profile else _Null():
+        ev0.record(stream)
+        for k in range(args.steps):
+            step(args.warmup + k)
+        ev1.record(stream)
+        ev1.synchronize()
+    torch.cuda.synchronize(dev)
+    t_ms = ev0.elapsed_time(ev1)
+    kt_total, kt_n = G.kernel_time(reset=True)
+    if world > 1:
+        tt = torch.tensor([t_ms], device=f"cuda:{dev}")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        torch.distributed.barrier()
+        t_ms = float(tt.item())
+    st = G.stats()
+    value = world * args.steps * g.m / (t_ms * 1e-3) / 1e9
+
+    if rank != 0:
+        if world > 1:
+            torch.distributed.barrier()
+            torch.distributed.destroy_process_group()
+        return
+
+    # ---------------- roofline of the dominant kernel (persistent Delta-stepping kernel)
+    used = [int(mine[(args.warmup + k) % len(mine)]) for k in range(args.steps)]
+    distinct = sorted(set(used))
+    balg = {}
+    out = np.empty(g.V, dtype=np.uint32 if g.wtype == "u32" else np.float32)
+    for s in distinct[:16]:
+        G.run(s, delta)
+        G.distances(out)
+        balg[s] = algorithmic_bytes(g, out.view(np.uint32), inf)
+    mean_b = float(np.mean([balg.get(s, balg[distinct[0]])[0] for s in used]))
+    kt_avg_ms = kt_total / max(kt_n, 1)
+    peak, peak_kind = measured_peak()
+    achieved = mean_b / (kt_avg_ms * 1e-3) / 1e9
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": load_traffic(args.config),
+            "peak_kind": peak_kind, "kernel": "k_delta_step (persistent)",
+            "kernel_ms_avg": round(kt_avg_ms, 4), "kernel_share_of_step": round(kt_total / t_ms, 4),
+            "alg_bytes_per_launch": int(mean_b)}
+
+    # ---------------- end-to-end through the public API, host buffers
+    e2e = None
+    if not args.no_e2e and not args.profile:
+        pinned = torch.empty(g.V, dtype=torch.int32).pin_memory()
+        ne = min(args.steps, 32)
+        for k in range(2):
+            G.run(int(mine[k % len(mine)]), delta)
+            G.distances(pinned)
+        t0 = time.perf_counter()
+        for k in range(ne):
+            G.run(int(mine[k % len(mine)]), delta)  # source id host -> device (launch argument)
+            G.distances(pinned)  # D2H of the result (synchronises)
+        te = time.perf_counter() - t0
+        e2e = {"value": round(ne * g.m / te / 1e9, 4), "unit": "GTEPS", "h2d_bytes_per_step": 8,
+               "d2h_bytes_per_step": 4 * g.V,
+               "note": "graph resident (uploaded+reordered once, like weights); per step: source id in, "
+                       "V distances out to pinned host memory; wall clock"}
+
+    cpu = None
+    if not args.no_cpu_baseline and not args.profile and world == 1:
+        cpu = cpu_baseline(g, sources)
+
+    line = {
+        "metric": METRIC, "value": round(value, 4), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(t_ms / args.steps, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32" if g.wtype == "u32" else "f32",
+        "data": "synthetic",
+        "config": {"workload": desc, "V": g.V, "m_edges": g.m, "arcs": g.A, "delta": delta,
+                   "reorder": reorder, "reorder_ms": reorder_ms, "sources": len(sources),
+                   "parallelism": f"replicas x{world} (sources sharded, graph replicated)",
+                   "l2": "inputs larger than L2 (arc array %.2f GB > 126 MB L2); dist re-initialised every step" % (8 * g.A / 1e9),
+                   "gen_s": round(t_gen, 1), "grid_ctas": st["grid_ctas"], "ring_slots": st["ring_slots"],
+                   "paper_v100_gteps_context": PAPER_V100.get(args.config)},
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": 3 * args.steps,
+        "clocks": sampler.summary() if not args.profile else None,
+        "last_run_stats": {k: st[k] for k in ("updates", "light_arcs", "heavy_arcs", "vertices_settled",
+                                              "stale_items", "hub_chunks", "buckets", "rescans", "reachable")},
+    }
+    print(json.dumps(line), flush=True)
+    G.close()
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        pass
+
+    def summary(self):
+        return None
+
+
+if __name__ == "__main__":
+    main()

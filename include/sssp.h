@@ -1,0 +1,170 @@
+/* sssp.h -- C-ABI of the B200-native bucket-aware asynchronous Delta-stepping
+ * SSSP library (libsssp.so, sm_100a).
+ *
+ * Method: Zhang et al., "A Bucket-aware Asynchronous Single-Source Shortest
+ * Path Algorithm on GPU", ICPP-W 2023. "P:n" cites line n of PAPER.md.
+ * Problem statement (Alg. 2 header P:1072-1075): given a graph
+ * G=(V,E,W), a starting vertex s and Delta, return the final shortest
+ * distance array dist.
+ *
+ * Conventions for every function:
+ *  - Return an sssp_status; never abort, never throw across the ABI. A
+ *    thread-local detail string is available from sssp_last_error().
+ *  - SSSP_ERR_CUDA is sticky for a handle: destroy it.
+ *  - All vertex ids at the API are the caller's ORIGINAL ids, also after
+ *    sssp_reorder (the relabelling is internal).
+ *  - Inputs are copied; the caller keeps ownership of every buffer it passes.
+ *    Output buffers are caller-allocated. The handle owns its device memory
+ *    until sssp_destroy.
+ *  - One host thread per handle at a time; handles are independent.
+ *  - Work is stream-ordered on the handle's stream (sssp_set_stream); only
+ *    sssp_graph_create, sssp_distances(HOST), sssp_get_stats and the export
+ *    helpers synchronise that stream.
+ */
+#ifndef SSSP_H
+#define SSSP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sssp_graph_s* sssp_graph_t; /* opaque, library-owned */
+
+typedef enum {
+    SSSP_OK = 0,
+    SSSP_ERR_INVALID_ARGUMENT = 1, /* bad size/pointer/id/Delta/CSR/weight */
+    SSSP_ERR_OUT_OF_MEMORY = 2,
+    SSSP_ERR_CUDA = 3,             /* CUDA runtime failure (sticky) */
+    SSSP_ERR_INVALID_STATE = 4,    /* e.g. sssp_distances before a successful sssp_run */
+    SSSP_ERR_OVERFLOW = 5,         /* a u32 distance reached 0xFFFFFFFF */
+    SSSP_ERR_INTERNAL = 6          /* scheduler safety cap hit (should not happen) */
+} sssp_status;
+
+typedef enum { SSSP_WEIGHT_U32 = 0, SSSP_WEIGHT_F32 = 1 } sssp_weight_type;
+typedef enum { SSSP_MEM_HOST = 0, SSSP_MEM_DEVICE = 1 } sssp_memory;
+
+/* Create a graph handle on CUDA device `device` from a CSR (DS-1):
+ *   row_offsets [V+1] int64: row[0]=0, non-decreasing, row[V]=A;
+ *   col_indices [A] uint32: each < V (arcs are directed; pass both directions
+ *                for an undirected graph, as the paper's figures do);
+ *   weights     [A] uint32, or float32 finite and >= 0 (-0.0 becomes +0.0).
+ * `where` says whether the three arrays are host or device pointers.
+ * 1 <= V < 2^31 and 0 <= A < 2^32 (arc offsets are kept 64-bit internally).
+ * cuda_stream: a cudaStream_t (NULL = legacy default stream).
+ * Validation runs on the device; the call synchronises the stream and returns
+ * SSSP_ERR_INVALID_ARGUMENT on any violation (*out untouched). */
+sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t num_vertices,
+                              int64_t num_arcs, const int64_t* row_offsets,
+                              const uint32_t* col_indices, const void* weights,
+                              sssp_weight_type wtype, sssp_memory where, void* cuda_stream);
+
+/* Property-driven reordering (PRO, PAPER §4.1, Fig. 4), on the GPU:
+ * relabel vertices by descending degree (ties by ascending original id) with
+ * a radix sort, permute the CSR, sort every adjacency by ascending weight
+ * (ties by ascending new id), and keep a heavy-edge offset per vertex in the
+ * row list (recomputed whenever Delta changes).
+ * Idempotent. Invalidates the previous sssp_run result. */
+sssp_status sssp_reorder(sssp_graph_t g);
+
+#define SSSP_PRO_DEGREE 1u /* relabel by descending degree */
+#define SSSP_PRO_WEIGHT 2u /* sort adjacencies by weight + heavy offsets */
+/* Ablation variant of sssp_reorder: flags = any subset of the two steps
+ * (0 restores nothing: reorder is one-way; 0 is a no-op). A graph with
+ * SSSP_PRO_WEIGHT uses the light/heavy split by offset; without it phases 1
+ * and 2 both scan whole adjacencies with a per-arc w < Delta predicate. */
+sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags);
+
+/* Single-source shortest paths from `source` (original id, 0 <= source < V)
+ * with bucket width `delta` (> 0; u32 graphs round it UP to an integer >= 1;
+ * f32 graphs round it to nearest binary32; +inf = one bucket, i.e. the
+ * Bellman-Ford end of Delta-stepping). Light arcs: w < Delta
+ * (P:265-266); bucket i holds distances in [i*Delta,(i+1)*Delta).
+ * Runs the bucket-aware asynchronous Delta-stepping of Alg. 2
+ * in one persistent cooperative kernel: phase 1 (light arcs, asynchronous,
+ * adaptive thread/warp/CTA bins),
+ * then fused phases 2&3 (heavy arcs + next bucket).
+ * Asynchronous w.r.t. the host (stream-ordered). The result is read with
+ * sssp_distances; overflow is reported there. */
+sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta);
+
+/* Copy the last run's distances (V elements of the graph's weight type, in
+ * ORIGINAL vertex order; unreachable = 0xFFFFFFFF for u32, +inf for f32) to
+ * `out` (host or device per `where`). HOST synchronises the stream.
+ * SSSP_ERR_INVALID_STATE if no successful run since create/reorder;
+ * SSSP_ERR_OVERFLOW if a u32 distance overflowed during the run. */
+sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory where);
+
+/* Free every resource of the handle. NULL-safe. */
+void sssp_destroy(sssp_graph_t g);
+
+/* ------------------------------------------------------------ helpers --- */
+const char* sssp_status_string(sssp_status s);
+const char* sssp_last_error(void); /* thread-local detail of the last failure */
+
+/* Make subsequent work on g use cuda_stream (a cudaStream_t; NULL = default). */
+sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream);
+
+/* Multi-source batch (the naturally sharded case of the north star): for
+ * i < n run sssp_run(sources[i], delta) and write the distances (original
+ * order) to the DEVICE buffer out_dev + i*ld elements (ld >= V). sources is a
+ * host array. Stream-ordered; no host synchronisation. */
+sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
+                           void* out_dev, int64_t ld);
+
+/* Counters of the last run (the work-efficiency metric of P:410-413 and
+ * updates = successful atomicMin writes; a valid update is one
+ * that writes the final distance, so valid = reachable - 1). Synchronises. */
+typedef struct sssp_stats {
+    uint64_t updates;          /* successful atomicMin improvements (total updates) */
+    uint64_t light_arcs;       /* light arcs relaxed in phase 1 */
+    uint64_t heavy_arcs;       /* heavy arcs relaxed in phase 2 */
+    uint64_t vertices_settled; /* phase-1 vertex items processed (non-stale) */
+    uint64_t stale_items;      /* phase-1 items skipped as stale */
+    uint64_t heavy_vertices;   /* phase-2 vertices whose heavy arcs were relaxed */
+    uint64_t hub_chunks;       /* 4096-arc chunks of vertices with > 4096 arcs in range */
+    uint64_t bin_thread;       /* vertices relaxed by the thread bin (< 32 arcs) */
+    uint64_t bin_warp;         /* ... warp bin (32..255) */
+    uint64_t bin_cta;          /* ... CTA bin (256..4096) */
+    uint64_t buckets;          /* phase-1 epochs run (buckets + reopenings) */
+    uint64_t rescans;          /* overflow fall-back rescans of dist[] */
+    uint64_t reachable;        /* vertices with a finite distance (filled by sssp_distances) */
+    uint32_t ring_slots;       /* K: bucket-queue ring size used */
+    uint32_t grid_ctas;        /* persistent grid size */
+    float run_ms;              /* device time of the last sssp_run (CUDA events) */
+    float reorder_ms;          /* device time of the last sssp_reorder */
+} sssp_stats;
+sssp_status sssp_get_stats(sssp_graph_t g, sssp_stats* s);
+
+/* Export the internal CSR (for parity tests against the paper's Fig. 4):
+ * rowlist [2V+1] int64 interleaved (start_v, heavy_v) + end with heavy offsets
+ * for `delta` (Fig. 4c layout); adj [A] uint32 internal ids;
+ * val [A] weights (4-byte, graph type); new2old [V] uint32 (identity if not
+ * reordered). Host pointers; any may be NULL. Synchronises. */
+sssp_status sssp_export_csr(sssp_graph_t g, double delta, int64_t* rowlist, uint32_t* adj,
+                            void* val, uint32_t* new2old);
+
+/* Tunables (defaults in brackets). Values are validated; takes effect at the
+ * next sssp_run. */
+typedef enum {
+    SSSP_PARAM_RING_SLOTS = 0,     /* K bucket queues, power of two in [4,64]; 0 = auto [0] */
+    SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
+    SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (1.25 V + 64Ki) [0] */
+    SSSP_PARAM_CLAIM_MAX = 3       /* max queue entries one CTA claims at once (1..256) [256] */
+} sssp_param;
+sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
+
+/* Device time of every persistent-kernel launch (CUDA events recorded around
+ * each cooperative launch on the handle's stream): *total_ms = sum since the
+ * last reset, *launches = how many. Synchronises on the pending events.
+ * reset != 0 zeroes the accumulators after reporting. */
+sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_t* launches, int reset);
+
+/* Library/device info: number of SMs of the handle's device. */
+int sssp_device_sm_count(sssp_graph_t g);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SSSP_H */

@@ -1,0 +1,61 @@
+// common.cuh -- small device helpers shared by the sm_100a kernels of libsssp.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#define SSSP_FULL_MASK 0xFFFFFFFFu
+
+namespace sssp {
+
+typedef unsigned long long u64;
+typedef uint32_t u32;
+typedef int64_t i64;
+
+// ---- loads / stores with explicit cache behaviour --------------------------
+// Arcs are streamed (read ~once per SSSP): evict-first in L1/L2.
+__device__ __forceinline__ uint2 ld_stream_u2(const uint2* p) { return __ldcs(p); }
+// Coherent (L2) load of mutable data (dist[], queue words).
+__device__ __forceinline__ u32 ld_cg(const u32* p) { return __ldcg(p); }
+__device__ __forceinline__ u64 ld_relaxed_u64(const u64* p) {
+  u64 v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ u32 ld_relaxed_u32(const u32* p) {
+  u32 v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
+  u32 v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(u64* p, u64 v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_u32(u32* p, u32 v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ u32 lanemask_lt() {
+  u32 m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+template <class T>
+__device__ __forceinline__ T warp_exclusive_scan(T x, T* total) {
+  const u32 lane = lane_id();
+  T v = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    T y = __shfl_up_sync(SSSP_FULL_MASK, v, o);
+    if (lane >= (u32)o) v += y;
+  }
+  *total = __shfl_sync(SSSP_FULL_MASK, v, 31);
+  return v - x;
+}
+
+}  // namespace sssp

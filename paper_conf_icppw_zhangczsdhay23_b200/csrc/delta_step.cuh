@@ -1,0 +1,798 @@
+// delta_step.cuh -- the persistent bucket-aware asynchronous Delta-stepping
+// kernel (sm_100a). One cooperative launch runs the whole bucket loop of
+// PAPER Alg. 2 on the device:
+//
+//   phase 1 (Alg. 2 l.6-9): asynchronous light-arc relaxation of the current
+//     bucket. CTAs pull batches of (v, d) entries from the bucket's queue,
+//     bin them by light degree l: l < 32 -> thread bin (arcs of
+//     a warp's small vertices spread over its lanes by a warp prefix sum,
+//     ranges staged in shared memory), 32 <= l < 256 -> warp per vertex,
+//     256 <= l <= 4096 -> CTA per vertex, l > 4096 -> ceil(l/4096) chunks any
+//     CTA may claim (reading R11). Improved vertices are pushed
+//     into the near queue (same bucket: visible at once, no level barrier,
+//     P:1100-1103) or a far bucket queue. The phase ends at quiescence:
+//     pend (pushed - completed) == 0 (manager/worker end rule).
+//   phases 2&3 (Alg. 2 l.13-19): after a grid barrier, heavy arcs
+//     of the bucket's settled vertices (entries with d == dist[v]) are relaxed
+//     once, hubs split into 4096-arc chunks; then the next non-empty bucket
+//     is chosen by the last CTA to arrive at the barrier (fused phase 3).
+//
+// Data (all device memory): dist[V] u32 (f32 as IEEE bits: order-preserving
+// for w >= 0, so one atomicMin.u32 serves both weight types, Alg. 1 l.3);
+// a ring of K bucket queues of packed u64 entries (d << 32 | v), each with one
+// 64-bit word (tail << 32 | pend) so a single atomicAdd both reserves slots and
+// counts pending work; entries are published by value (SENTINEL = empty).
+// Pushes beyond the ring horizon or beyond a queue's capacity are dropped and
+// recorded in far_min; the scheduler then rebuilds the ring from dist[]
+// (topological rescan, as the paper's phase 3 loops over all V, Alg. 2 l.13).
+#pragma once
+#include "common.cuh"
+
+namespace sssp {
+
+constexpr int DS_THREADS = 256;
+constexpr int DS_WARPS = DS_THREADS / 32;
+constexpr u32 BIN_WARP = 32;     // beta
+constexpr u32 BIN_CTA = 256;     // alpha
+constexpr u32 HUB_CHUNK = 4096;
+constexpr int UNROLL = 4;
+constexpr u64 SENTINEL = ~0ULL;
+constexpr u32 NONE = 0xFFFFFFFFu;
+constexpr u32 CHUNK_FLAG = 0x80000000u;
+
+enum : u32 {
+  MODE_PHASE1 = 0,
+  MODE_PHASE2 = 1,
+  MODE_DONE = 2,
+  MODE_RESCAN_CLEAR = 3,
+  MODE_RESCAN_FILL = 4,
+  MODE_SWEEP_LIGHT = 5,
+  MODE_SWEEP_HEAVY = 6
+};
+enum : u32 { ERR_OVERFLOW = 1, ERR_INTERNAL = 2 };
+enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5 };
+enum : u32 { SRC_QUEUE = 0, SRC_STATIC = 1, SRC_HUB = 2, SRC_SWEEP = 3 };
+
+enum {
+  ST_UPDATES = 0,
+  ST_LIGHT,
+  ST_HEAVY,
+  ST_SETTLED,
+  ST_STALE,
+  ST_HEAVYV,
+  ST_CHUNKS,
+  ST_BIN_T,
+  ST_BIN_W,
+  ST_BIN_C,
+  ST_N
+};
+
+struct Ctl {
+  u32 cur, lim, mode, far_min;
+  u32 p2_begin, p2_end, p2_head, err;
+  u32 bar_count, bar_gen, epochs, rescans;
+  u32 rescan_base, changed, sweep_first, sweeps;
+  u64 hub_word;
+  u32 hub_head, pad3;
+};
+
+struct Params {
+  const longlong2* rowp;  // [V+1] {start, heavy}
+  const uint2* arcs;      // [A] {dst, wbits}
+  u32* dist;              // [V]
+  u32* xd;                // [V] sweep fall-back: distance at last light expansion
+  Ctl* ctl;
+  u64* word;              // [K]
+  u32* head;              // [K]
+  u32* p2;                // [K]
+  u64* items;             // [K * cap]
+  u64* hub_items;         // [hub_cap]
+  unsigned long long* stats;  // [ST_N]
+  u32 V, K, kmask, cap, hub_cap;
+  u32 delta_u;       // u32 graphs: integer Delta >= 1
+  float inv_delta;   // f32 graphs: fl32(1/Delta)
+  u32 delta_bits;    // light iff wbits < delta_bits
+  u32 claim_max;
+};
+
+struct Smem {
+  u64 items[DS_THREADS];
+  i64 wl_beg[DS_THREADS];
+  u32 wl_len[DS_THREADS];
+  u32 wl_d[DS_THREADS];
+  i64 cl_beg[DS_THREADS];
+  u32 cl_len[DS_THREADS];
+  u32 cl_d[DS_THREADS];
+  i64 sb_beg[DS_WARPS][32];
+  u32 sb_off[DS_WARPS][32];
+  u32 sb_d[DS_WARPS][32];
+  unsigned long long st[ST_N];
+  u32 wl_n, wl_next, cl_n;
+  u32 claim_h, claim_n, claim_src;
+  // control snapshot
+  u32 mode, cur, lim, p2_begin, p2_end, sweep_first;
+};
+
+// ---------------------------------------------------------------- helpers --
+template <bool F32>
+__device__ __forceinline__ u32 relax_add(u32 d, u32 w, u32* err) {
+  if (F32) {
+    return __float_as_uint(__fadd_rn(__uint_as_float(d), __uint_as_float(w)));  // Alg. 1 l.1
+  } else {
+    u64 s = (u64)d + w;
+    if (s >= (u64)NONE) {
+      atomicOr(err, ERR_OVERFLOW);
+      return NONE;  // treated as "no improvement"
+    }
+    return (u32)s;
+  }
+}
+
+template <bool F32>
+__device__ __forceinline__ u32 bucket_of(const Params& p, u32 d) {
+  if (F32) {
+    u32 b = __float2uint_rz(__fmul_rn(__uint_as_float(d), p.inv_delta));
+    return b >= NONE ? NONE - 1 : b;
+  } else {
+    return d / p.delta_u;
+  }
+}
+
+__device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
+  u32 s = __reduce_add_sync(SSSP_FULL_MASK, x);
+  if (lane_id() == 0 && s) atomicAdd(&sm.st[k], (unsigned long long)s);
+}
+
+// Push (v, nd) into the queue of bucket(nd). Must be called by all 32 lanes.
+// nearb != NONE (sweep fall-back): improvements landing in bucket nearb are
+// not queued; they mark v for the next sweep instead.
+template <bool F32>
+__device__ __forceinline__ void warp_push(const Params& p, Smem& sm, u32 lim, bool want, u32 v,
+                                          u32 nd, u32 nearb) {
+  const u32 any = __ballot_sync(SSSP_FULL_MASK, want);
+  if (!any) return;
+  if (lane_id() == (u32)(__ffs(any) - 1)) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)__popc(any));
+  u32 x = 0;
+  bool ok = false;
+  if (want) {
+    x = bucket_of<F32>(p, nd);
+    if (x == nearb) {
+      st_relaxed_u32(p.xd + v, NONE);
+      st_relaxed_u32(&p.ctl->changed, 1u);
+    } else {
+      ok = x <= lim;
+      if (!ok) atomicMin(&p.ctl->far_min, x);  // beyond the ring horizon: rescan later
+    }
+  }
+  const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
+  if (ok) {
+    const u32 s = x & p.kmask;
+    const u32 peers = __match_any_sync(m, s);
+    const u32 leader = __ffs(peers) - 1;
+    const u32 cnt = __popc(peers);
+    u64 old = 0;
+    if (lane_id() == leader) old = atomicAdd(p.word + s, ((u64)cnt << 32) | cnt);
+    old = __shfl_sync(peers, old, leader);
+    const u32 idx = (u32)(old >> 32) + __popc(peers & lanemask_lt());
+    if (idx < p.cap) {
+      st_relaxed_u64(p.items + (u64)s * p.cap + idx, ((u64)nd << 32) | v);
+    } else {  // queue full: undo the pending count, recover by rescan
+      atomicAdd(p.word + s, ~0ULL);
+      atomicMin(&p.ctl->far_min, x);
+    }
+  }
+}
+
+// Relax UNROLL arcs per thread (independent loads in flight: arcs, then dist
+// probes, then atomics). PH 1 = light arcs, PH 2 = heavy arcs; without PRO the
+// light/heavy split is a per-arc predicate (the divergence PRO removes).
+template <bool F32, bool PRO, int PH>
+__device__ __forceinline__ void relax_group(const Params& p, Smem& sm, u32 lim, u32 nearb,
+                                            const i64 (&idx)[UNROLL], const bool (&valid)[UNROLL],
+                                            const u32 (&d)[UNROLL]) {
+  uint2 a[UNROLL];
+  u32 nd[UNROLL];
+  bool want[UNROLL];
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) a[k] = valid[k] ? ld_stream_u2(p.arcs + idx[k]) : make_uint2(0, 0);
+  u32 cur[UNROLL];
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) {
+    bool take = valid[k];
+    if (!PRO) take = take && ((PH == 1) ? (a[k].y < p.delta_bits) : (a[k].y >= p.delta_bits));
+    want[k] = take;
+    nd[k] = take ? relax_add<F32>(d[k], a[k].y, &p.ctl->err) : NONE;
+    cur[k] = take ? ld_cg(p.dist + a[k].x) : 0u;
+  }
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) {
+    want[k] = want[k] && nd[k] < cur[k];  // check before the atomic (Alg. 1 l.2)
+    if (want[k]) want[k] = nd[k] < atomicMin(p.dist + a[k].x, nd[k]);  // Alg. 1 l.3
+  }
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) warp_push<F32>(p, sm, lim, want[k], a[k].x, nd[k], nearb);
+}
+
+// Range of an item for phase PH: PRO -> light [start, heavy) / heavy [heavy, end);
+// no PRO -> the whole adjacency (predicate per arc).
+template <bool PRO, int PH>
+__device__ __forceinline__ void item_range(const Params& p, u32 v, i64& b, i64& e) {
+  const longlong2 r = p.rowp[v];
+  if (PRO && PH == 1) {
+    b = r.x;
+    e = r.y;
+  } else {
+    e = p.rowp[v + 1].x;
+    b = (PRO && PH == 2) ? r.y : r.x;
+  }
+}
+
+// ------------------------------------------------------------ batch -------
+// Process the CTA's claimed items (one per thread; has = thread holds one).
+// src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
+// phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
+// into the current bucket, hubs stay in the CTA bin).
+template <bool F32, bool PRO, int PH>
+__device__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 lim, u32 src,
+                              u32 slot) {
+  const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const bool sweep = src == SRC_SWEEP;
+  const u32 nearb = sweep ? sm.cur : NONE;
+  bool small = false;
+  i64 beg = 0;
+  u32 len = 0, d = 0;
+  u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0;
+  if (has) {
+    const u32 lo = (u32)it, hi = (u32)(it >> 32);
+    bool is_chunk = (lo & CHUNK_FLAG) != 0;
+    const u32 v = lo & ~CHUNK_FLAG;
+    bool live = false;
+    if (is_chunk) {
+      // Chunk items in the phase-2 static range are phase-1 work already done.
+      live = !(PH == 2 && src == SRC_STATIC);
+      if (live) {
+        i64 rb, re;
+        item_range<PRO, PH>(p, v, rb, re);
+        beg = rb + (i64)hi * HUB_CHUNK;
+        len = (u32)min((i64)HUB_CHUNK, re - beg);
+        d = ld_cg(p.dist + v);  // current distance: a valid path length (<= spawning d)
+        c_arcs = len;
+        u32 i = atomicAdd(&sm.cl_n, 1u);
+        sm.cl_beg[i] = beg;
+        sm.cl_len[i] = len;
+        sm.cl_d[i] = d;
+      }
+    } else {
+      const u32 cd = ld_cg(p.dist + v);
+      d = hi;
+      live = (PH == 1) ? (d <= cd) : (d == cd);  // stale filter / settled-final filter
+      if (!live) {
+        c_stale = (PH == 1);
+      } else {
+        c_settled = 1;
+        i64 rb, re;
+        item_range<PRO, PH>(p, v, rb, re);
+        const i64 l = re - rb;
+        c_arcs = (u32)min(l, (i64)0xFFFFFFFF);
+        if (l > (i64)HUB_CHUNK && !sweep) {  // hub: ceil(l/4096) chunks any CTA may claim
+          const u32 nc = (u32)((l + HUB_CHUNK - 1) / HUB_CHUNK);
+          c_chunks = nc;
+          c_arcs = 0;  // counted when the chunks run
+          u64* word = (PH == 1) ? p.word + slot : &p.ctl->hub_word;
+          u64* q = (PH == 1) ? p.items + (u64)slot * p.cap : p.hub_items;
+          const u32 qcap = (PH == 1) ? p.cap : p.hub_cap;
+          const u32 base = (u32)(atomicAdd(word, ((u64)nc << 32) | nc) >> 32);
+          for (u32 c = 0; c < nc; ++c) {
+            if (base + c < qcap) {
+              st_relaxed_u64(q + base + c, ((u64)c << 32) | CHUNK_FLAG | v);
+            } else {
+              atomicAdd(word, ~0ULL);
+              if (PH == 1)
+                atomicMin(&p.ctl->far_min, sm.cur);  // lost phase-1 work: rescan this bucket
+              else
+                atomicOr(&p.ctl->err, ERR_INTERNAL);
+            }
+          }
+        } else if (l >= (i64)BIN_CTA) {
+          u32 i = atomicAdd(&sm.cl_n, 1u);
+          sm.cl_beg[i] = rb;
+          sm.cl_len[i] = (u32)l;
+          sm.cl_d[i] = d;
+        } else if (l >= (i64)BIN_WARP) {
+          u32 i = atomicAdd(&sm.wl_n, 1u);
+          sm.wl_beg[i] = rb;
+          sm.wl_len[i] = (u32)l;
+          sm.wl_d[i] = d;
+        } else if (l > 0) {
+          small = true;
+          beg = rb;
+          len = (u32)l;
+        }
+      }
+    }
+  }
+  // ---- stats (warp-aggregated)
+  st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
+  if (PH == 1) st_add(sm, ST_STALE, c_stale);
+  st_add(sm, PH == 1 ? ST_LIGHT : ST_HEAVY, c_arcs);
+  st_add(sm, ST_CHUNKS, c_chunks);
+  st_add(sm, ST_BIN_T, small ? 1u : 0u);
+
+  // ---- thread bin: a warp's small vertices, arcs spread by a warp prefix sum
+  {
+    u32 total;
+    const u32 off = warp_exclusive_scan(small ? len : 0u, &total);
+    if (total) {
+      sm.sb_beg[w][lane] = beg;
+      sm.sb_off[w][lane] = off;
+      sm.sb_d[w][lane] = d;
+      __syncwarp();
+      for (u32 j0 = 0; j0 < total; j0 += 32 * UNROLL) {
+        i64 idx[UNROLL];
+        bool valid[UNROLL];
+        u32 dd[UNROLL];
+#pragma unroll
+        for (int k = 0; k < UNROLL; ++k) {
+          const u32 j = j0 + k * 32 + lane;
+          valid[k] = j < total;
+          u32 o = 0;  // owner: last lane with sb_off <= j
+#pragma unroll
+          for (u32 step = 16; step; step >>= 1)
+            if (sm.sb_off[w][o + step] <= j) o += step;
+          idx[k] = sm.sb_beg[w][o] + (j - sm.sb_off[w][o]);
+          dd[k] = sm.sb_d[w][o];
+        }
+        relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
+      }
+      __syncwarp();
+    }
+  }
+  __syncthreads();
+  // ---- warp bin: one warp per vertex (32 <= l < 256)
+  if (tid == 0) {
+    sm.st[ST_BIN_W] += sm.wl_n;
+    sm.st[ST_BIN_C] += sm.cl_n;
+  }
+  for (;;) {
+    u32 i = 0;
+    if (lane == 0) i = atomicAdd(&sm.wl_next, 1u);
+    i = __shfl_sync(SSSP_FULL_MASK, i, 0);
+    if (i >= sm.wl_n) break;
+    const i64 b = sm.wl_beg[i];
+    const u32 l = sm.wl_len[i];
+    const u32 dv = sm.wl_d[i];
+    for (u32 j0 = 0; j0 < l; j0 += 32 * UNROLL) {
+      i64 idx[UNROLL];
+      bool valid[UNROLL];
+      u32 dd[UNROLL];
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        const u32 j = j0 + k * 32 + lane;
+        valid[k] = j < l;
+        idx[k] = b + j;
+        dd[k] = dv;
+      }
+      relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
+    }
+  }
+  // ---- CTA bin: the whole CTA per vertex / chunk (256 <= l <= 4096)
+  const u32 ncl = sm.cl_n;
+  for (u32 i = 0; i < ncl; ++i) {
+    const i64 b = sm.cl_beg[i];
+    const u32 l = sm.cl_len[i];
+    const u32 dv = sm.cl_d[i];
+    for (u32 j0 = 0; j0 < l; j0 += DS_THREADS * UNROLL) {
+      i64 idx[UNROLL];
+      bool valid[UNROLL];
+      u32 dd[UNROLL];
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        const u32 j = j0 + k * DS_THREADS + tid;
+        valid[k] = j < l;
+        idx[k] = b + j;
+        dd[k] = dv;
+      }
+      relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    sm.wl_n = 0;
+    sm.wl_next = 0;
+    sm.cl_n = 0;
+  }
+}
+
+// --------------------------------------------------------- grid barrier ---
+// Last CTA to arrive runs the serial scheduler step (fused phase 3).
+__device__ void decide(const Params& p, u32 which) {
+  volatile Ctl* c = p.ctl;
+  volatile u64* word = p.word;
+  volatile u32* head = p.head;
+  volatile u32* p2 = p.p2;
+  const u32 K = p.K;
+  if (which == SYNC_P1) {
+    const u32 cur = c->cur, s = cur & p.kmask;
+    if (c->far_min <= cur) {  // phase-1 work was dropped (queue full): sweep fall-back
+      c->changed = 0;
+      c->sweep_first = 1;
+      c->sweeps = c->sweeps + 1;
+      c->mode = MODE_SWEEP_LIGHT;
+      return;
+    }
+    const u64 wv = word[s];
+    const u32 tail = min((u32)(wv >> 32), p.cap);
+    const u32 b = p2[s];
+    c->p2_begin = b;
+    c->p2_end = tail;
+    c->p2_head = b;
+    c->hub_word = (u64)(tail - b);  // pending = static entries; chunks add to it
+    c->hub_head = 0;
+    c->mode = MODE_PHASE2;
+  } else if (which == SYNC_P2) {
+    const u32 cur = c->cur, s = cur & p.kmask;
+    p2[s] = c->p2_end;
+    const u32 fm = c->far_min;
+    if ((u32)word[s] != 0) {  // f32: a heavy relaxation rounded into bucket cur
+      if (fm <= cur) {
+        c->changed = 0;
+        c->sweep_first = 1;
+        c->sweeps = c->sweeps + 1;
+        c->mode = MODE_SWEEP_LIGHT;
+      } else {
+        c->mode = MODE_PHASE1;
+        c->epochs = c->epochs + 1;
+      }
+      return;
+    }
+    u32 nxt = NONE;
+    for (u32 x = cur + 1; x <= c->lim && x != NONE; ++x)
+      if ((u32)(word[x & p.kmask] >> 32) != 0) {
+        nxt = x;
+        break;
+      }
+    if (nxt == NONE && fm == NONE) {
+      c->mode = MODE_DONE;
+      return;
+    }
+    if (fm <= nxt) {  // a dropped push precedes the ring's next bucket
+      c->rescan_base = fm;
+      c->mode = MODE_RESCAN_CLEAR;
+      return;
+    }
+    word[s] = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
+    head[s] = 0;
+    p2[s] = 0;
+    const u64 lim = (u64)cur + K - 1;  // excludes slot s: it is reset now
+    c->lim = (u32)min(lim, (u64)NONE - 1);
+    c->cur = nxt;
+    c->mode = MODE_PHASE1;
+    c->epochs = c->epochs + 1;
+  } else if (which == SYNC_RC) {
+    for (u32 s = 0; s < K; ++s) {
+      word[s] = 0;
+      head[s] = 0;
+      p2[s] = 0;
+    }
+    const u32 r = c->rescan_base;
+    c->far_min = NONE;
+    c->cur = r;
+    c->lim = (u32)min((u64)r + K - 1, (u64)NONE - 1);
+    c->mode = MODE_RESCAN_FILL;
+  } else if (which == SYNC_RF) {
+    c->mode = MODE_PHASE1;
+    c->epochs = c->epochs + 1;
+    c->rescans = c->rescans + 1;
+  } else {  // SYNC_SL / SYNC_SH: sweep fall-back of bucket cur
+    if (c->changed) {  // something improved inside bucket cur: sweep light arcs again
+      c->changed = 0;
+      c->sweep_first = 0;
+      c->mode = MODE_SWEEP_LIGHT;
+    } else if (which == SYNC_SL) {
+      c->mode = MODE_SWEEP_HEAVY;
+    } else {  // bucket cur is final; rebuild the ring from dist[] for what follows
+      c->rescan_base = c->cur + 1;
+      c->mode = MODE_RESCAN_CLEAR;
+    }
+  }
+}
+
+__device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    Ctl* c = p.ctl;
+    const u32 gen = ld_acquire_u32(&c->bar_gen);
+    __threadfence();
+    const u32 arrived = atomicAdd(&c->bar_count, 1u);
+    if (arrived == gridDim.x - 1) {
+      c->bar_count = 0;
+      __threadfence();
+      decide(p, which);
+      __threadfence();
+      atomicAdd(&c->bar_gen, 1u);
+    } else {
+      u32 ns = 32;
+      while (ld_acquire_u32(&c->bar_gen) == gen) {
+        __nanosleep(ns);
+        if (ns < 256) ns <<= 1;
+      }
+    }
+    __threadfence();
+    volatile Ctl* vc = c;
+    sm.mode = vc->mode;
+    sm.cur = vc->cur;
+    sm.lim = vc->lim;
+    sm.p2_begin = vc->p2_begin;
+    sm.p2_end = vc->p2_end;
+    sm.sweep_first = vc->sweep_first;
+  }
+  __syncthreads();
+}
+
+// ------------------------------------------------------------ phases ------
+template <bool F32, bool PRO>
+__device__ void phase1(const Params& p, Smem& sm) {
+  const u32 slot = sm.cur & p.kmask, lim = sm.lim;
+  u64* q = p.items + (u64)slot * p.cap;
+  const u32 G = gridDim.x;
+  for (;;) {
+    if (threadIdx.x == 0) {
+      u32 n = 0, h = 0, ns = 32;
+      for (;;) {
+        const u64 wv = ld_relaxed_u64(p.word + slot);
+        const u32 tail = min((u32)(wv >> 32), p.cap);
+        h = ld_relaxed_u32(p.head + slot);
+        if (h < tail) {
+          const u32 avail = tail - h;
+          u32 want = (avail + G - 1) / G;
+          want = max(want, 16u);
+          want = min(want, p.claim_max);
+          n = min(avail, want);
+          if (atomicCAS(p.head + slot, h, h + n) == h) break;
+          continue;
+        }
+        if ((u32)wv == 0) {  // quiescent: nothing pending anywhere
+          n = 0;
+          break;
+        }
+        __nanosleep(ns);
+        if (ns < 512) ns <<= 1;
+      }
+      sm.claim_n = n;
+      sm.claim_h = h;
+    }
+    __syncthreads();
+    const u32 n = sm.claim_n;
+    if (n == 0) break;
+    const u32 h = sm.claim_h;
+    u64 it = SENTINEL;
+    const bool has = threadIdx.x < n;
+    if (has) {
+      u64* e = q + h + threadIdx.x;
+      u32 ns = 16;
+      while ((it = ld_relaxed_u64(e)) == SENTINEL) {  // reserved, not yet written
+        __nanosleep(ns);
+        if (ns < 256) ns <<= 1;
+      }
+    }
+    process_batch<F32, PRO, 1>(p, sm, it, has, lim, SRC_QUEUE, slot);
+    if (threadIdx.x == 0) atomicAdd(p.word + slot, (u64)0 - (u64)n);  // completion
+  }
+}
+
+template <bool F32, bool PRO>
+__device__ void phase2(const Params& p, Smem& sm) {
+  const u32 slot = sm.cur & p.kmask, lim = sm.lim;
+  u64* q = p.items + (u64)slot * p.cap;
+  const u32 p2e = sm.p2_end;
+  const u32 G = gridDim.x;
+  const u32 span = sm.p2_end - sm.p2_begin;
+  const u32 CL = min(max((span + G - 1) / G, 16u), p.claim_max);
+  Ctl* c = p.ctl;
+  for (;;) {
+    if (threadIdx.x == 0) {
+      u32 n = 0, h = 0, src = 0, ns = 32;
+      for (;;) {
+        if (ld_relaxed_u32(&c->p2_head) < p2e) {
+          h = atomicAdd(&c->p2_head, CL);
+          if (h < p2e) {
+            n = min(CL, p2e - h);
+            src = 1;
+            break;
+          }
+        }
+        const u64 wv = ld_relaxed_u64(&c->hub_word);
+        const u32 tail = min((u32)(wv >> 32), p.hub_cap);
+        const u32 hh = ld_relaxed_u32(&c->hub_head);
+        if (hh < tail) {
+          const u32 nn = min(tail - hh, 2u);
+          if (atomicCAS(&c->hub_head, hh, hh + nn) == hh) {
+            h = hh;
+            n = nn;
+            src = 2;
+            break;
+          }
+          continue;
+        }
+        if ((u32)wv == 0) {
+          n = 0;
+          break;
+        }
+        __nanosleep(ns);
+        if (ns < 512) ns <<= 1;
+      }
+      sm.claim_n = n;
+      sm.claim_h = h;
+      sm.claim_src = src;
+    }
+    __syncthreads();
+    const u32 n = sm.claim_n;
+    if (n == 0) break;
+    const u32 h = sm.claim_h, src = sm.claim_src;
+    u64 it = SENTINEL;
+    const bool has = threadIdx.x < n;
+    if (has) {
+      if (src == SRC_STATIC) {
+        u64* e = q + h + threadIdx.x;
+        it = ld_relaxed_u64(e);
+        st_relaxed_u64(e, SENTINEL);  // recycle the queue entry
+      } else {
+        u64* e = p.hub_items + h + threadIdx.x;
+        u32 ns = 16;
+        while ((it = ld_relaxed_u64(e)) == SENTINEL) {
+          __nanosleep(ns);
+          if (ns < 256) ns <<= 1;
+        }
+        st_relaxed_u64(e, SENTINEL);
+      }
+    }
+    process_batch<F32, PRO, 2>(p, sm, it, has, lim, src, slot);
+    if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
+  }
+}
+
+// Rescan stage 1: clear every queue entry still holding a value.
+__device__ void rescan_clear(const Params& p) {
+  const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
+  const i64 nt = (i64)gridDim.x * blockDim.x;
+  for (u32 s = 0; s < p.K; ++s) {
+    const u32 tail = min((u32)(ld_relaxed_u64(p.word + s) >> 32), p.cap);
+    u64* q = p.items + (u64)s * p.cap;
+    for (i64 i = t; i < tail; i += nt) st_relaxed_u64(q + i, SENTINEL);
+  }
+}
+
+// Rescan stage 2: every unsettled vertex (bucket(dist) >= base) is pushed anew.
+template <bool F32>
+__device__ void rescan_fill(const Params& p, Smem& sm) {
+  const u32 base = sm.cur, lim = sm.lim;
+  const i64 t0 = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL;
+  const i64 nt = (i64)gridDim.x * blockDim.x;
+  for (i64 b = t0; b < p.V; b += nt) {
+    const i64 v = b + lane_id();
+    bool want = false;
+    u32 d = NONE;
+    if (v < p.V) {
+      d = ld_cg(p.dist + v);
+      want = d != (F32 ? 0x7F800000u : NONE) && bucket_of<F32>(p, d) >= base;
+    }
+    warp_push<F32>(p, sm, lim, want, (u32)v, d, NONE);
+  }
+}
+
+// Sweep fall-back for a bucket whose queue lost work (capacity): Bellman-Ford
+// style sweeps over all v with bucket(dist[v]) == cur until nothing in the
+// bucket improves (light arcs; xd[] skips vertices unchanged since their last
+// expansion), then one sweep over heavy arcs. Always makes progress.
+template <bool F32, bool PRO, int PH>
+__device__ void sweep(const Params& p, Smem& sm) {
+  const u32 cur = sm.cur, lim = sm.lim;
+  const bool first = sm.sweep_first != 0;
+  const u32 inf = F32 ? 0x7F800000u : NONE;
+  for (i64 base = (i64)blockIdx.x * DS_THREADS; base < p.V; base += (i64)gridDim.x * DS_THREADS) {
+    const i64 v = base + threadIdx.x;
+    bool has = false;
+    u64 it = SENTINEL;
+    if (v < p.V) {
+      const u32 d = ld_cg(p.dist + v);
+      if (d != inf && bucket_of<F32>(p, d) == cur) {
+        if (PH == 1) {
+          if (first || d < ld_cg(p.xd + v)) {
+            st_relaxed_u32(p.xd + v, d);
+            has = true;
+          }
+        } else {
+          has = true;
+        }
+        it = ((u64)d << 32) | (u64)v;
+      }
+    }
+    process_batch<F32, PRO, PH>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);
+  }
+}
+
+template <bool F32, bool PRO>
+__global__ void __launch_bounds__(DS_THREADS, 2) k_delta_step(Params p) {
+  __shared__ Smem sm;
+  if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
+  if (threadIdx.x == 0) {
+    sm.wl_n = 0;
+    sm.wl_next = 0;
+    sm.cl_n = 0;
+    volatile Ctl* vc = p.ctl;
+    sm.mode = vc->mode;
+    sm.cur = vc->cur;
+    sm.lim = vc->lim;
+    sm.p2_begin = vc->p2_begin;
+    sm.p2_end = vc->p2_end;
+    sm.sweep_first = vc->sweep_first;
+  }
+  __syncthreads();
+  for (;;) {
+    const u32 mode = sm.mode;
+    if (mode == MODE_DONE) break;
+    if (mode == MODE_PHASE1) {
+      phase1<F32, PRO>(p, sm);
+      grid_barrier(p, sm, SYNC_P1);
+    } else if (mode == MODE_PHASE2) {
+      phase2<F32, PRO>(p, sm);
+      grid_barrier(p, sm, SYNC_P2);
+    } else if (mode == MODE_RESCAN_CLEAR) {
+      rescan_clear(p);
+      grid_barrier(p, sm, SYNC_RC);
+    } else if (mode == MODE_RESCAN_FILL) {
+      rescan_fill<F32>(p, sm);
+      grid_barrier(p, sm, SYNC_RF);
+    } else if (mode == MODE_SWEEP_LIGHT) {
+      sweep<F32, PRO, 1>(p, sm);
+      grid_barrier(p, sm, SYNC_SL);
+    } else {
+      sweep<F32, PRO, 2>(p, sm);
+      grid_barrier(p, sm, SYNC_SH);
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x < ST_N && sm.st[threadIdx.x]) atomicAdd(p.stats + threadIdx.x, sm.st[threadIdx.x]);
+}
+
+// ------------------------------------------------------------- init -------
+__global__ void k_fill_u32(u32* __restrict__ a, i64 n, u32 v) {
+  i64 i = (i64)blockIdx.x * blockDim.x + threadIdx.x;
+  i64 stride = (i64)gridDim.x * blockDim.x;
+  for (; i < n; i += stride) a[i] = v;
+}
+
+// Alg. 2 l.1-3: dist[s] = 0, bucket 0 queue holds (s, 0), counters reset.
+__global__ void k_seed(Params p, u32 src) {
+  const u32 t = threadIdx.x;
+  for (u32 s = t; s < p.K; s += blockDim.x) {
+    p.word[s] = 0;
+    p.head[s] = 0;
+    p.p2[s] = 0;
+  }
+  if (t < ST_N) p.stats[t] = 0;
+  __syncthreads();
+  if (t == 0) {
+    p.dist[src] = 0;
+    p.items[0] = (u64)src;  // (d=0 << 32) | src in bucket 0, slot 0
+    p.word[0] = (1ULL << 32) | 1ULL;
+    Ctl* c = p.ctl;
+    c->cur = 0;
+    c->lim = p.K - 1;
+    c->mode = MODE_PHASE1;
+    c->far_min = NONE;
+    c->p2_begin = c->p2_end = c->p2_head = 0;
+    c->err = 0;
+    c->bar_count = 0;
+    c->epochs = 1;
+    c->rescans = 0;
+    c->rescan_base = 0;
+    c->changed = 0;
+    c->sweep_first = 0;
+    c->sweeps = 0;
+    c->hub_word = 0;
+    c->hub_head = 0;
+  }
+}
+
+}  // namespace sssp

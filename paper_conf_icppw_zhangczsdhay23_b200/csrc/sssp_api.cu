@@ -1,0 +1,722 @@
+// sssp_api.cu -- C-ABI runtime of libsssp.so (see include/sssp.h).
+// Host side: validation, device memory, stream-ordered launches. Every step
+// of the SSSP path runs in the kernels of pro.cuh / sort.cuh / delta_step.cuh.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/sssp.h"
+#include "delta_step.cuh"
+#include "pro.cuh"
+#include "sort.cuh"
+
+using namespace sssp;
+
+// --------------------------------------------------------------- errors ---
+static thread_local std::string g_last_error;
+
+static sssp_status fail(sssp_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return s;
+}
+
+struct sssp_graph_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int num_sms = 0;
+  i64 V = 0, A = 0;
+  sssp_weight_type wtype = SSSP_WEIGHT_U32;
+  longlong2* rowp = nullptr;  // [V+1] {start, heavy}
+  uint2* arcs = nullptr;      // [A]
+  u32 maxw_bits = 0;
+  u32* old2new = nullptr;  // null until PRO_DEGREE
+  u32* new2old = nullptr;
+  std::vector<u32> h_old2new;  // host copy: source mapping without a sync per run
+  unsigned pro_flags = 0;
+  bool heavy_valid = false;
+  u32 heavy_bits = 0;
+  // run state
+  u32* dist = nullptr;
+  u32* xd = nullptr;
+  Ctl* ctl = nullptr;
+  u64* word = nullptr;
+  u32* head = nullptr;
+  u32* p2 = nullptr;
+  u64* items = nullptr;
+  u64* hub_items = nullptr;
+  unsigned long long* stats = nullptr;
+  u32 K_alloc = 0, cap_alloc = 0, hub_cap = 0;
+  u32 K_used = 0;
+  bool need_full_reset = true;
+  bool have_result = false;
+  bool sticky_cuda = false;
+  int grid_ctas = 0;
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  // per-launch timing of the persistent kernel (sssp_kernel_time)
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev_pending;
+  double kt_total_ms = 0.0;
+  int64_t kt_launches = 0;
+  bool run_timed = false, reorder_timed = false;
+  // params
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = 256;
+};
+
+#define CU(call)                                                                       \
+  do {                                                                                 \
+    cudaError_t e_ = (call);                                                           \
+    if (e_ != cudaSuccess) {                                                           \
+      if (g) g->sticky_cuda = true;                                                    \
+      return fail(e_ == cudaErrorMemoryAllocation ? SSSP_ERR_OUT_OF_MEMORY : SSSP_ERR_CUDA, \
+                  "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));  \
+    }                                                                                  \
+  } while (0)
+
+static unsigned grid_for(i64 n, int threads = 256) {
+  i64 b = (n + threads - 1) / threads;
+  return (unsigned)std::max<i64>(1, std::min<i64>(b, 148 * 32));
+}
+
+static sssp_status check_handle(sssp_graph_t g) {
+  if (!g) return fail(SSSP_ERR_INVALID_ARGUMENT, "null graph handle");
+  if (g->sticky_cuda) return fail(SSSP_ERR_CUDA, "handle is in a failed CUDA state; destroy it");
+  return SSSP_OK;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    cudaGetDevice(&prev);
+    if (prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// --------------------------------------------------------------- create ---
+extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t V, int64_t A,
+                                         const int64_t* row, const uint32_t* col,
+                                         const void* weights, sssp_weight_type wtype,
+                                         sssp_memory where, void* cuda_stream) {
+  sssp_graph_s* g = nullptr;
+  if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+  if (V < 1 || V >= 0x7FFFFFFFLL) return fail(SSSP_ERR_INVALID_ARGUMENT, "V=%lld out of [1, 2^31-1)", (long long)V);
+  if (A < 0 || A >= 0xFFFFFFFFLL) return fail(SSSP_ERR_INVALID_ARGUMENT, "A=%lld out of [0, 2^32-1)", (long long)A);
+  if (!row || (A > 0 && (!col || !weights))) return fail(SSSP_ERR_INVALID_ARGUMENT, "null CSR pointer");
+  if (wtype != SSSP_WEIGHT_U32 && wtype != SSSP_WEIGHT_F32) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad weight type");
+  if (where != SSSP_MEM_HOST && where != SSSP_MEM_DEVICE) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad memory kind");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
+    return fail(SSSP_ERR_INVALID_ARGUMENT, "CUDA device %d not available", device);
+  DeviceGuard dg(device);
+  g = new (std::nothrow) sssp_graph_s();
+  if (!g) return fail(SSSP_ERR_OUT_OF_MEMORY, "host allocation failed");
+  g->device = device;
+  g->stream = (cudaStream_t)cuda_stream;
+  g->V = V;
+  g->A = A;
+  g->wtype = wtype;
+  cudaDeviceProp prop;
+  sssp_status st = SSSP_OK;
+  auto bail = [&](sssp_status s) {
+    sssp_destroy(g);
+    return s;
+  };
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return bail(fail(SSSP_ERR_CUDA, "cudaGetDeviceProperties"));
+  g->num_sms = prop.multiProcessorCount;
+  const cudaMemcpyKind kind = where == SSSP_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  i64* d_row = nullptr;
+  u32 *d_col = nullptr, *d_w = nullptr, *d_flags = nullptr;
+  do {
+    cudaStream_t s = g->stream;
+#define CG(call)                                                                        \
+    {                                                                                   \
+      cudaError_t e_ = (call);                                                          \
+      if (e_ != cudaSuccess) {                                                          \
+        st = fail(e_ == cudaErrorMemoryAllocation ? SSSP_ERR_OUT_OF_MEMORY : SSSP_ERR_CUDA, \
+                  "create: %s: %s", #call, cudaGetErrorString(e_));                     \
+        break;                                                                          \
+      }                                                                                 \
+    }
+    CG(cudaMalloc(&g->rowp, sizeof(longlong2) * (V + 1)));
+    CG(cudaMalloc(&g->arcs, sizeof(uint2) * std::max<i64>(A, 1)));
+    CG(cudaMalloc(&g->dist, sizeof(u32) * V));
+    CG(cudaMalloc(&g->xd, sizeof(u32) * V));
+    CG(cudaMalloc(&g->ctl, sizeof(Ctl)));
+    CG(cudaMalloc(&g->stats, sizeof(unsigned long long) * ST_N));
+    CG(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
+    CG(cudaMemsetAsync(g->stats, 0, sizeof(unsigned long long) * ST_N, s));
+    for (int i = 0; i < 4; ++i) CG(cudaEventCreate(&g->ev[i]));
+    CG(cudaMallocAsync(&d_row, sizeof(i64) * (V + 1), s));
+    CG(cudaMallocAsync(&d_flags, sizeof(u32) * 2, s));
+    CG(cudaMemsetAsync(d_flags, 0, sizeof(u32) * 2, s));
+    CG(cudaMemcpyAsync(d_row, row, sizeof(i64) * (V + 1), kind, s));
+    if (A > 0) {
+      CG(cudaMallocAsync(&d_col, sizeof(u32) * A, s));
+      CG(cudaMallocAsync(&d_w, sizeof(u32) * A, s));
+      CG(cudaMemcpyAsync(d_col, col, sizeof(u32) * A, kind, s));
+      CG(cudaMemcpyAsync(d_w, weights, sizeof(u32) * A, kind, s));
+    }
+    k_check_rows<<<grid_for(V), 256, 0, s>>>(d_row, V, A, d_flags);
+    k_rows_to_rowp<<<grid_for(V + 1), 256, 0, s>>>(d_row, V, g->rowp);
+    if (A > 0)
+      k_pack_arcs<<<grid_for(A), 256, 0, s>>>(d_col, d_w, A, (u32)V, wtype == SSSP_WEIGHT_F32,
+                                               g->arcs, d_flags, d_flags + 1);
+    CG(cudaGetLastError());
+    u32 flags[2] = {0, 0};
+    CG(cudaMemcpyAsync(flags, d_flags, sizeof flags, cudaMemcpyDeviceToHost, s));
+    CG(cudaFreeAsync(d_row, s));
+    d_row = nullptr;
+    CG(cudaFreeAsync(d_flags, s));
+    d_flags = nullptr;
+    if (d_col) CG(cudaFreeAsync(d_col, s));
+    d_col = nullptr;
+    if (d_w) CG(cudaFreeAsync(d_w, s));
+    d_w = nullptr;
+    CG(cudaStreamSynchronize(s));
+    if (flags[0]) {
+      st = fail(SSSP_ERR_INVALID_ARGUMENT, "invalid CSR:%s%s%s%s", (flags[0] & 1) ? " row[0]!=0 or row[V]!=A" : "",
+                (flags[0] & 2) ? " row offsets decrease" : "", (flags[0] & 4) ? " col index >= V" : "",
+                (flags[0] & 8) ? " weight negative/NaN/inf" : "");
+      break;
+    }
+    g->maxw_bits = flags[1];
+#undef CG
+  } while (0);
+  if (st != SSSP_OK) {
+    if (d_row) cudaFree(d_row);
+    if (d_col) cudaFree(d_col);
+    if (d_w) cudaFree(d_w);
+    if (d_flags) cudaFree(d_flags);
+    return bail(st);
+  }
+  *out = g;
+  return SSSP_OK;
+}
+
+extern "C" void sssp_destroy(sssp_graph_t g) {
+  if (!g) return;
+  DeviceGuard dg(g->device);
+  if (g->stream) cudaStreamSynchronize(g->stream);
+  else cudaDeviceSynchronize();
+  void* ptrs[] = {g->rowp, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->word,
+                  g->head, g->p2, g->items, g->hub_items, g->stats};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  for (auto& e : g->ev)
+    if (e) cudaEventDestroy(e);
+  for (auto& e : g->ev_pool) cudaEventDestroy(e);
+  for (auto& pr : g->ev_pending) {
+    cudaEventDestroy(pr.first);
+    cudaEventDestroy(pr.second);
+  }
+  cudaGetLastError();  // do not leak a sticky error to the caller's context
+  delete g;
+}
+
+extern "C" const char* sssp_status_string(sssp_status s) {
+  switch (s) {
+    case SSSP_OK: return "SSSP_OK";
+    case SSSP_ERR_INVALID_ARGUMENT: return "SSSP_ERR_INVALID_ARGUMENT";
+    case SSSP_ERR_OUT_OF_MEMORY: return "SSSP_ERR_OUT_OF_MEMORY";
+    case SSSP_ERR_CUDA: return "SSSP_ERR_CUDA";
+    case SSSP_ERR_INVALID_STATE: return "SSSP_ERR_INVALID_STATE";
+    case SSSP_ERR_OVERFLOW: return "SSSP_ERR_OVERFLOW";
+    case SSSP_ERR_INTERNAL: return "SSSP_ERR_INTERNAL";
+  }
+  return "SSSP_UNKNOWN_STATUS";
+}
+
+extern "C" const char* sssp_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream) {
+  sssp_status s = check_handle(g);
+  if (s) return s;
+  g->stream = (cudaStream_t)cuda_stream;
+  return SSSP_OK;
+}
+
+extern "C" int sssp_device_sm_count(sssp_graph_t g) { return g ? g->num_sms : 0; }
+
+extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
+  sssp_status s = check_handle(g);
+  if (s) return s;
+  switch (p) {
+    case SSSP_PARAM_RING_SLOTS:
+      if (v != 0 && (v < 4 || v > 64 || (v & (v - 1)))) return fail(SSSP_ERR_INVALID_ARGUMENT, "ring slots must be 0 or a power of two in [4,64]");
+      g->p_ring = v;
+      return SSSP_OK;
+    case SSSP_PARAM_CTAS_PER_SM:
+      if (v < 0 || v > 32) return fail(SSSP_ERR_INVALID_ARGUMENT, "ctas per SM in [0,32]");
+      g->p_ctas = v;
+      return SSSP_OK;
+    case SSSP_PARAM_SLOT_CAPACITY:
+      if (v < 0 || v > 0x7FFFFFFFLL || (v != 0 && v < 4096)) return fail(SSSP_ERR_INVALID_ARGUMENT, "slot capacity 0 or in [4096, 2^31)");
+      g->p_cap = v;
+      return SSSP_OK;
+    case SSSP_PARAM_CLAIM_MAX:
+      if (v < 1 || v > DS_THREADS) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,256]");
+      g->p_claim = v;
+      return SSSP_OK;
+  }
+  return fail(SSSP_ERR_INVALID_ARGUMENT, "unknown parameter %d", (int)p);
+}
+
+// --------------------------------------------------------------- reorder --
+template <int NF>
+static sssp_status radix_pass(sssp_graph_t g, Fields<NF>& a, Fields<NF>& b, int kf, i64 n, int sh,
+                              u32* hist, u32* tmp) {
+  cudaStream_t s = g->stream;
+  const u32 ntiles = (u32)((n + RS_TILE - 1) / RS_TILE);
+  k_rs_hist<<<ntiles, RS_THREADS, 0, s>>>(a.f[kf], n, sh, hist, ntiles);
+  scan_exclusive_rec<u32>(hist, hist, (i64)256 * ntiles, tmp, s);
+  k_rs_scatter<NF><<<ntiles, RS_THREADS, 0, s>>>(a, b, kf, n, sh, hist, ntiles);
+  std::swap(a, b);
+  CU(cudaGetLastError());
+  return SSSP_OK;
+}
+
+static int bits_for(u64 maxv) {
+  int b = 0;
+  while (b < 64 && (maxv >> b) != 0) ++b;
+  return b;
+}
+
+extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (flags & ~(SSSP_PRO_DEGREE | SSSP_PRO_WEIGHT)) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad PRO flags 0x%x", flags);
+  if ((flags & ~g->pro_flags) == 0) return SSSP_OK;  // idempotent
+  if (g->pro_flags != 0)
+    return fail(SSSP_ERR_INVALID_STATE, "graph already reordered with flags 0x%x", g->pro_flags);
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  const i64 V = g->V, A = g->A;
+  const bool deg = flags & SSSP_PRO_DEGREE, wsort = flags & SSSP_PRO_WEIGHT;
+  CU(cudaEventRecord(g->ev[2], s));
+  // temporaries
+  const i64 nmax = std::max<i64>(std::max(V, A), 1);
+  const i64 ntiles_max = (nmax + RS_TILE - 1) / RS_TILE;
+  const i64 hist_n = 256 * ntiles_max;
+  u32 *hist = nullptr, *tmp = nullptr, *f[6] = {}, *dmax = nullptr;
+  u64 *ndeg = nullptr, *stmp = nullptr;
+  CU(cudaMallocAsync(&hist, sizeof(u32) * hist_n, s));
+  CU(cudaMallocAsync(&tmp, sizeof(u32) * scan_tmp_elems(hist_n), s));
+  CU(cudaMallocAsync(&dmax, sizeof(u32), s));
+  CU(cudaMemsetAsync(dmax, 0, sizeof(u32), s));
+  if (deg) {
+    // a1: stable radix sort of (maxdeg - deg, id) -> new2old (desc degree, asc id)
+    if (!g->new2old) CU(cudaMalloc(&g->new2old, sizeof(u32) * V));
+    if (!g->old2new) CU(cudaMalloc(&g->old2new, sizeof(u32) * V));
+    u32 *key0, *key1, *id1;
+    CU(cudaMallocAsync(&key0, sizeof(u32) * V, s));
+    CU(cudaMallocAsync(&key1, sizeof(u32) * V, s));
+    CU(cudaMallocAsync(&id1, sizeof(u32) * V, s));
+    k_max_degree<<<grid_for(V), 256, 0, s>>>(g->rowp, V, dmax);
+    k_degree_keys<<<grid_for(V), 256, 0, s>>>(g->rowp, V, dmax, key0, g->new2old);
+    u32 maxdeg = 0;
+    CU(cudaMemcpyAsync(&maxdeg, dmax, sizeof(u32), cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    Fields<2> a{{key0, g->new2old}}, b{{key1, id1}};
+    const int nb = bits_for(maxdeg);
+    for (int sh = 0; sh < nb; sh += 8) {
+      st = radix_pass<2>(g, a, b, 0, V, sh, hist, tmp);
+      if (st) return st;
+    }
+    if (a.f[1] != g->new2old) CU(cudaMemcpyAsync(g->new2old, a.f[1], sizeof(u32) * V, cudaMemcpyDeviceToDevice, s));
+    CU(cudaMallocAsync(&ndeg, sizeof(u64) * (V + 1), s));
+    CU(cudaMallocAsync(&stmp, sizeof(u64) * scan_tmp_elems(V), s));
+    k_invert_perm<<<grid_for(V), 256, 0, s>>>(g->new2old, g->rowp, V, g->old2new, ndeg);
+    scan_exclusive_rec<u64>(ndeg, ndeg, V, stmp, s);  // new row starts
+    CU(cudaFreeAsync(key0, s));
+    CU(cudaFreeAsync(key1, s));
+    CU(cudaFreeAsync(id1, s));
+    CU(cudaGetLastError());
+  }
+  if (A > 0) {
+    // a2+a3: one stable LSD radix sort of all arcs by (new src, w, new dst)
+    for (int i = 0; i < 6; ++i) CU(cudaMallocAsync(&f[i], sizeof(u32) * A, s));
+    k_expand_arcs<<<grid_for((i64)V * 32), 256, 0, s>>>(g->rowp, g->arcs, V, deg ? g->old2new : nullptr,
+                                                       f[0], f[1], f[2]);
+    CU(cudaGetLastError());
+    Fields<3> a{{f[0], f[1], f[2]}}, b{{f[3], f[4], f[5]}};
+    const int vb = bits_for((u64)(V - 1));
+    if (wsort) {
+      for (int sh = 0; sh < vb; sh += 8)
+        if ((st = radix_pass<3>(g, a, b, 2, A, sh, hist, tmp))) return st;
+      const int wb = bits_for(g->maxw_bits);
+      for (int sh = 0; sh < wb; sh += 8)
+        if ((st = radix_pass<3>(g, a, b, 1, A, sh, hist, tmp))) return st;
+    }
+    if (deg || wsort)
+      for (int sh = 0; sh < vb; sh += 8)
+        if ((st = radix_pass<3>(g, a, b, 0, A, sh, hist, tmp))) return st;
+    k_pack_sorted<<<grid_for(A), 256, 0, s>>>(a.f[1], a.f[2], A, g->arcs);
+    CU(cudaGetLastError());
+    for (int i = 0; i < 6; ++i) CU(cudaFreeAsync(f[i], s));
+  }
+  if (deg) {
+    k_set_rowp<<<grid_for(V + 1), 256, 0, s>>>(ndeg, V, A, g->rowp);
+    CU(cudaFreeAsync(ndeg, s));
+    CU(cudaFreeAsync(stmp, s));
+  }
+  CU(cudaFreeAsync(hist, s));
+  CU(cudaFreeAsync(tmp, s));
+  CU(cudaFreeAsync(dmax, s));
+  CU(cudaEventRecord(g->ev[3], s));
+  CU(cudaGetLastError());
+  if (deg) {
+    g->h_old2new.resize(V);
+    CU(cudaMemcpyAsync(g->h_old2new.data(), g->old2new, sizeof(u32) * V, cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+  }
+  g->pro_flags |= flags;
+  g->heavy_valid = false;
+  g->have_result = false;
+  g->reorder_timed = true;
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_reorder(sssp_graph_t g) {
+  return sssp_reorder_ex(g, SSSP_PRO_DEGREE | SSSP_PRO_WEIGHT);
+}
+
+// ------------------------------------------------------------------ run ---
+struct DeltaParams {
+  u32 delta_u, delta_bits;
+  float inv;
+  double ahead;  // max weight / Delta (buckets a heavy push can skip ahead)
+};
+
+static sssp_status delta_params(sssp_graph_t g, double delta, DeltaParams* dp) {
+  if (std::isnan(delta) || delta <= 0.0) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta must be > 0 (got %g)", delta);
+  if (g->wtype == SSSP_WEIGHT_U32) {
+    double c = std::ceil(delta);
+    dp->delta_u = (std::isinf(delta) || c >= 4294967295.0) ? 0xFFFFFFFFu : (u32)std::max(1.0, c);
+    dp->delta_bits = dp->delta_u;
+    dp->inv = 0.f;
+    dp->ahead = (double)g->maxw_bits / dp->delta_u;
+  } else {
+    float df = (float)delta;
+    if (df <= 0.f) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta rounds to 0 in binary32");
+    u32 bits;
+    memcpy(&bits, &df, 4);
+    dp->delta_bits = bits;
+    dp->delta_u = 1;
+    dp->inv = std::isinf(df) ? 0.f : (float)(1.0 / (double)df);
+    float mw;
+    memcpy(&mw, &g->maxw_bits, 4);
+    dp->ahead = std::isinf(df) ? 0.0 : (double)mw / (double)df;
+  }
+  return SSSP_OK;
+}
+
+static sssp_status ensure_run_buffers(sssp_graph_t g, u32 K, u32 cap) {
+  cudaStream_t s = g->stream;
+  const u32 hub_cap = (u32)std::min<i64>(g->A / 2048 + 4096, 0x7FFFFFFF);
+  if (K > g->K_alloc || cap != g->cap_alloc) {
+    if (g->items) CU(cudaFree(g->items));
+    if (g->word) CU(cudaFree(g->word));
+    if (g->head) CU(cudaFree(g->head));
+    if (g->p2) CU(cudaFree(g->p2));
+    g->items = nullptr;
+    g->word = nullptr;
+    g->head = nullptr;
+    g->p2 = nullptr;
+    CU(cudaMalloc(&g->items, sizeof(u64) * (size_t)K * cap));
+    CU(cudaMalloc(&g->word, sizeof(u64) * K));
+    CU(cudaMalloc(&g->head, sizeof(u32) * K));
+    CU(cudaMalloc(&g->p2, sizeof(u32) * K));
+    g->K_alloc = K;
+    g->cap_alloc = cap;
+    g->need_full_reset = true;
+  }
+  if (!g->hub_items) {
+    CU(cudaMalloc(&g->hub_items, sizeof(u64) * hub_cap));
+    g->hub_cap = hub_cap;
+    g->need_full_reset = true;
+  }
+  if (g->need_full_reset) {
+    CU(cudaMemsetAsync(g->items, 0xFF, sizeof(u64) * (size_t)g->K_alloc * g->cap_alloc, s));
+    CU(cudaMemsetAsync(g->hub_items, 0xFF, sizeof(u64) * g->hub_cap, s));
+    g->need_full_reset = false;
+  }
+  return SSSP_OK;
+}
+
+typedef void (*ds_kernel_t)(Params);
+static ds_kernel_t pick_kernel(bool f32, bool pro) {
+  if (f32) return pro ? k_delta_step<true, true> : k_delta_step<true, false>;
+  return pro ? k_delta_step<false, true> : k_delta_step<false, false>;
+}
+
+static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParams& dp, bool timed) {
+  cudaStream_t s = g->stream;
+  const bool pro = (g->pro_flags & SSSP_PRO_WEIGHT) != 0;
+  const bool f32 = g->wtype == SSSP_WEIGHT_F32;
+  // a4: heavy offsets for this Delta (only with weight-sorted adjacencies)
+  if (pro && (!g->heavy_valid || g->heavy_bits != dp.delta_bits)) {
+    k_heavy_offsets<<<grid_for(g->V), 256, 0, s>>>(g->rowp, g->arcs, g->V, dp.delta_bits);
+    CU(cudaGetLastError());
+    g->heavy_valid = true;
+    g->heavy_bits = dp.delta_bits;
+  }
+  // ring size: enough slots for the farthest heavy push (+ the recycled slot)
+  u32 K = (u32)g->p_ring;
+  if (K == 0) {
+    double need = std::ceil(dp.ahead) + 3.0;
+    K = 8;
+    while (K < need && K < 32) K <<= 1;
+  }
+  u32 cap = (u32)g->p_cap;
+  if (cap == 0) cap = (u32)std::min<i64>(g->V + g->V / 4 + 65536, 0x7FFFFFFF);
+  sssp_status st = ensure_run_buffers(g, K, cap);
+  if (st) return st;
+  g->K_used = K;
+  ds_kernel_t kern = pick_kernel(f32, pro);
+  int per_sm = 0;
+  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, DS_THREADS, 0));
+  if (per_sm < 1) return fail(SSSP_ERR_INTERNAL, "persistent kernel cannot be resident");
+  if (g->p_ctas > 0) per_sm = std::min<int>(per_sm, (int)g->p_ctas);
+  g->grid_ctas = per_sm * g->num_sms;
+  Params p;
+  p.rowp = g->rowp;
+  p.arcs = g->arcs;
+  p.dist = g->dist;
+  p.xd = g->xd;
+  p.ctl = g->ctl;
+  p.word = g->word;
+  p.head = g->head;
+  p.p2 = g->p2;
+  p.items = g->items;
+  p.hub_items = g->hub_items;
+  p.stats = g->stats;
+  p.V = (u32)g->V;
+  p.K = K;
+  p.kmask = K - 1;
+  p.cap = cap;
+  p.hub_cap = g->hub_cap;
+  p.delta_u = dp.delta_u;
+  p.inv_delta = dp.inv;
+  p.delta_bits = dp.delta_bits;
+  p.claim_max = (u32)g->p_claim;
+  // a5: init (Alg. 2 l.1-3)
+  k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
+  k_seed<<<1, 64, 0, s>>>(p, src_internal);
+  CU(cudaGetLastError());
+  cudaEvent_t e0, e1;
+  for (int i = 0; i < 2; ++i) {
+    cudaEvent_t e;
+    if (g->ev_pool.empty()) {
+      CU(cudaEventCreate(&e));
+    } else {
+      e = g->ev_pool.back();
+      g->ev_pool.pop_back();
+    }
+    (i ? e1 : e0) = e;
+  }
+  g->ev_pending.emplace_back(e0, e1);
+  CU(cudaEventRecord(e0, s));
+  if (timed) CU(cudaEventRecord(g->ev[0], s));
+  void* args[] = {&p};
+  CU(cudaLaunchCooperativeKernel((const void*)kern, dim3(g->grid_ctas), dim3(DS_THREADS), args, 0, s));
+  if (timed) CU(cudaEventRecord(g->ev[1], s));
+  CU(cudaEventRecord(e1, s));
+  g->run_timed = timed;
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (source < 0 || source >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source %lld out of range", (long long)source);
+  DeltaParams dp;
+  if ((st = delta_params(g, delta, &dp))) return st;
+  DeviceGuard dg(g->device);
+  const u32 src = g->h_old2new.empty() ? (u32)source : g->h_old2new[source];
+  g->have_result = false;
+  if ((st = launch_run(g, src, dp, true))) return st;
+  g->have_result = true;
+  return SSSP_OK;
+}
+
+// ------------------------------------------------------------ results -----
+static sssp_status check_run_errors(sssp_graph_t g) {
+  Ctl c;
+  CU(cudaMemcpyAsync(&c, g->ctl, sizeof c, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaStreamSynchronize(g->stream));
+  if (c.err & ERR_INTERNAL) {
+    g->need_full_reset = true;
+    return fail(SSSP_ERR_INTERNAL, "scheduler queue overflow");
+  }
+  if (c.err & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory where) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+  if (where != SSSP_MEM_HOST && where != SSSP_MEM_DEVICE) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad memory kind");
+  if (!g->have_result) return fail(SSSP_ERR_INVALID_STATE, "no successful sssp_run since create/reorder");
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  u32* dst = (u32*)out;
+  u32* tmp = nullptr;
+  if (where == SSSP_MEM_HOST) CU(cudaMallocAsync(&tmp, sizeof(u32) * g->V, s));
+  k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, tmp ? tmp : dst);
+  CU(cudaGetLastError());
+  if (tmp) {
+    CU(cudaMemcpyAsync(dst, tmp, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
+    CU(cudaFreeAsync(tmp, s));
+  }
+  return check_run_errors(g);
+}
+
+extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
+                                      void* out_dev, int64_t ld) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (n < 0 || (n > 0 && (!sources || !out_dev)) || ld < g->V)
+    return fail(SSSP_ERR_INVALID_ARGUMENT, "bad batch arguments");
+  DeltaParams dp;
+  if ((st = delta_params(g, delta, &dp))) return st;
+  for (i64 i = 0; i < n; ++i)
+    if (sources[i] < 0 || sources[i] >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source[%lld] out of range", (long long)i);
+  DeviceGuard dg(g->device);
+  std::vector<u32> src(n);
+  for (i64 i = 0; i < n; ++i) src[i] = g->h_old2new.empty() ? (u32)sources[i] : g->h_old2new[sources[i]];
+  for (i64 i = 0; i < n; ++i) {
+    g->have_result = false;
+    if ((st = launch_run(g, src[i], dp, i == n - 1))) return st;
+    g->have_result = true;
+    k_output<<<grid_for(g->V), 256, 0, g->stream>>>(g->dist, g->old2new, g->V, (u32*)out_dev + (size_t)i * ld);
+    CU(cudaGetLastError());
+  }
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_get_stats(sssp_graph_t g, sssp_stats* out) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  memset(out, 0, sizeof *out);
+  unsigned long long h[ST_N];
+  Ctl c;
+  unsigned long long* cnt = nullptr;
+  CU(cudaMallocAsync(&cnt, sizeof(unsigned long long), s));
+  CU(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), s));
+  k_count_finite<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, g->wtype == SSSP_WEIGHT_F32 ? 0x7F800000u : 0xFFFFFFFFu, cnt);
+  unsigned long long reach = 0;
+  CU(cudaMemcpyAsync(&reach, cnt, sizeof reach, cudaMemcpyDeviceToHost, s));
+  CU(cudaMemcpyAsync(h, g->stats, sizeof h, cudaMemcpyDeviceToHost, s));
+  CU(cudaMemcpyAsync(&c, g->ctl, sizeof c, cudaMemcpyDeviceToHost, s));
+  CU(cudaFreeAsync(cnt, s));
+  CU(cudaStreamSynchronize(s));
+  out->updates = h[ST_UPDATES];
+  out->light_arcs = h[ST_LIGHT];
+  out->heavy_arcs = h[ST_HEAVY];
+  out->vertices_settled = h[ST_SETTLED];
+  out->stale_items = h[ST_STALE];
+  out->heavy_vertices = h[ST_HEAVYV];
+  out->hub_chunks = h[ST_CHUNKS];
+  out->bin_thread = h[ST_BIN_T];
+  out->bin_warp = h[ST_BIN_W];
+  out->bin_cta = h[ST_BIN_C];
+  out->buckets = c.epochs;
+  out->rescans = c.rescans + c.sweeps;
+  out->reachable = g->have_result ? reach : 0;
+  out->ring_slots = g->K_used;
+  out->grid_ctas = (u32)g->grid_ctas;
+  if (g->run_timed) CU(cudaEventElapsedTime(&out->run_ms, g->ev[0], g->ev[1]));
+  if (g->reorder_timed) CU(cudaEventElapsedTime(&out->reorder_ms, g->ev[2], g->ev[3]));
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_export_csr(sssp_graph_t g, double delta, int64_t* rowlist, uint32_t* adj,
+                                       void* val, uint32_t* new2old) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  DeltaParams dp;
+  if ((st = delta_params(g, delta, &dp))) return st;
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  const i64 V = g->V, A = g->A;
+  if (rowlist) {
+    std::vector<longlong2> r(V + 1);
+    if (g->pro_flags & SSSP_PRO_WEIGHT) {
+      longlong2* tmp = nullptr;
+      CU(cudaMallocAsync(&tmp, sizeof(longlong2) * (V + 1), s));
+      CU(cudaMemcpyAsync(tmp, g->rowp, sizeof(longlong2) * (V + 1), cudaMemcpyDeviceToDevice, s));
+      k_heavy_offsets<<<grid_for(V), 256, 0, s>>>(tmp, g->arcs, V, dp.delta_bits);
+      CU(cudaGetLastError());
+      CU(cudaMemcpyAsync(r.data(), tmp, sizeof(longlong2) * (V + 1), cudaMemcpyDeviceToHost, s));
+      CU(cudaFreeAsync(tmp, s));
+    } else {
+      CU(cudaMemcpyAsync(r.data(), g->rowp, sizeof(longlong2) * (V + 1), cudaMemcpyDeviceToHost, s));
+      for (auto& x : r) x.y = x.x;  // no weight order: no heavy offset
+    }
+    CU(cudaStreamSynchronize(s));
+    for (i64 i = 0; i < V; ++i) {
+      rowlist[2 * i] = r[i].x;
+      rowlist[2 * i + 1] = r[i].y;
+    }
+    rowlist[2 * V] = r[V].x;
+  }
+  if ((adj || val) && A > 0) {
+    std::vector<uint2> a(A);
+    CU(cudaMemcpyAsync(a.data(), g->arcs, sizeof(uint2) * A, cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    for (i64 i = 0; i < A; ++i) {
+      if (adj) adj[i] = a[i].x;
+      if (val) ((u32*)val)[i] = a[i].y;
+    }
+  }
+  if (new2old) {
+    if (g->new2old) {
+      CU(cudaMemcpyAsync(new2old, g->new2old, sizeof(u32) * V, cudaMemcpyDeviceToHost, s));
+      CU(cudaStreamSynchronize(s));
+    } else {
+      for (i64 i = 0; i < V; ++i) new2old[i] = (u32)i;
+    }
+  }
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_t* launches, int reset) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  DeviceGuard dg(g->device);
+  for (auto& pr : g->ev_pending) {
+    CU(cudaEventSynchronize(pr.second));
+    float ms = 0.f;
+    CU(cudaEventElapsedTime(&ms, pr.first, pr.second));
+    g->kt_total_ms += ms;
+    g->kt_launches += 1;
+    g->ev_pool.push_back(pr.first);
+    g->ev_pool.push_back(pr.second);
+  }
+  g->ev_pending.clear();
+  if (total_ms) *total_ms = g->kt_total_ms;
+  if (launches) *launches = g->kt_launches;
+  if (reset) {
+    g->kt_total_ms = 0.0;
+    g->kt_launches = 0;
+  }
+  return SSSP_OK;
+}

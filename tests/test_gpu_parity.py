@@ -1,0 +1,327 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the CPU oracle, element by
+element, on seeded inputs. u32 distances must be bit-exact; f32 distances are
+bit-exact too (the f32 result is the unique min over left-to-right binary32
+path sums), which is stricter than north_star's 1e-6."""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+INF = oracle.INF_U32
+
+
+@pytest.fixture(scope="module")
+def sssp():
+    import torch
+
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import __graft_entry__
+
+    __graft_entry__.build_cuda()
+    import paper_conf_icppw_zhangczsdhay23_b200 as m
+
+    return m
+
+
+def bits(a):
+    return np.ascontiguousarray(a).view(np.uint32)
+
+
+def assert_same(got, exp, what=""):
+    gb, eb = bits(got), bits(exp)
+    if not np.array_equal(gb, eb):
+        bad = np.flatnonzero(gb != eb)
+        raise AssertionError(f"{what}: {len(bad)} mismatches; first {bad[:8].tolist()} "
+                             f"got {gb[bad[:8]].tolist()} exp {eb[bad[:8]].tolist()}")
+
+
+def csr_from_arcs(V, arcs, wdtype=np.uint32):
+    arcs = sorted(arcs, key=lambda a: a[0])
+    row = np.zeros(V + 1, dtype=np.int64)
+    for u, _, _ in arcs:
+        row[u + 1] += 1
+    row = np.cumsum(row).astype(np.int64)
+    col = np.array([a[1] for a in arcs], dtype=np.uint32)
+    w = np.array([a[2] for a in arcs], dtype=wdtype)
+    return row, col, w
+
+
+# ------------------------------------------------------ paper examples ----
+def test_fig4_pro_on_gpu(sssp, golden):
+    g = golden("fig4_pro.json")
+    arcs = []
+    for u, v, w in g["edges"]:
+        arcs += [(u, v, w), (v, u, w)]
+    arcs.sort(key=lambda a: (a[0], a[1]))
+    for wd in (np.uint32, np.float32):
+        row, col, w = csr_from_arcs(g["V"], arcs, wd)
+        with sssp.Graph(row, col, w) as G:
+            G.reorder()
+            ex = G.export_csr(g["delta"])
+            assert ex["new2old"].tolist() == g["new2old"]
+            assert ex["rowlist"].tolist() == g["rowlist"]
+            assert ex["adj"].tolist() == g["adj"]
+            assert ex["val"].astype(np.int64).tolist() == g["val"]
+            for d, rl in g["rowlist_by_delta"].items():
+                assert G.export_csr(float(d))["rowlist"].tolist() == rl
+            for s in range(g["V"]):
+                assert G.sssp(s, g["delta"]).astype(np.int64).tolist() == g["dist"][s]
+
+
+def test_fig1_distances_on_gpu(sssp, golden):
+    g = golden("fig1_csr.json")
+    adj = g["adj_printed_rows_0_4"] + g["adj_rows_5_7_by_symmetry"]
+    val = g["val_printed_rows_0_4"] + [g["w67"] if x == "w67" else x for x in g["val_rows_5_7_by_symmetry"]]
+    row = np.array(g["row"], np.int64)
+    col, w = np.array(adj, np.uint32), np.array(val, np.uint32)
+    for reorder in (False, True):
+        with sssp.Graph(row, col, w) as G:
+            if reorder:
+                G.reorder()
+            assert G.sssp(0, g["delta"]).tolist() == g["dist_from_0"]
+
+
+# ------------------------------------------------------------- random -----
+CASES = [
+    # scale, ef, weights, deltas
+    (10, 16, "u32", (1, 7, 32, 1e9, float("inf"))),
+    (13, 16, "u32", (16, 100)),
+    (10, 16, "f32", (0.01, 0.1, 1.0, float("inf"))),
+    (13, 8, "f32", (0.1,)),
+]
+
+
+@pytest.mark.parametrize("scale,ef,wt,deltas", CASES)
+@pytest.mark.parametrize("flags", [3, 0, 1, 2])
+def test_kronecker_parity(sssp, scale, ef, wt, deltas, flags):
+    g = gen.kronecker(scale, ef, seed=100 + scale, weights=wt)
+    srcs = gen.sample_sources(g, 3, seed=scale)
+    exp = {int(s): oracle.dijkstra(g.row, g.col, g.w, int(s)) for s in srcs}
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if flags:
+            G.reorder(flags)
+        for d in deltas:
+            for s in srcs:
+                assert_same(G.sssp(int(s), d), exp[int(s)], f"s{scale} {wt} flags={flags} delta={d} src={s}")
+
+
+def test_grid_many_buckets(sssp):
+    g = gen.grid(300, 200, p=0.2, seed=5)
+    s = int(gen.sample_sources(g, 1, seed=1)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    for reorder in (True, False):
+        with sssp.Graph(g.row, g.col, g.w) as G:
+            if reorder:
+                G.reorder()
+            for d in (50, 400, 1600):
+                assert_same(G.sssp(s, d), exp, f"grid reorder={reorder} delta={d}")
+                st = G.stats()
+                assert st["buckets"] >= int(exp[exp != INF].max()) // max(d, 1) // 2
+
+
+# ---------------------------------------------------------- edge cases ----
+def test_single_vertex_and_no_arcs(sssp):
+    with sssp.Graph(np.zeros(2, np.int64), np.zeros(0, np.uint32), np.zeros(0, np.uint32)) as G:
+        assert G.sssp(0, 5).tolist() == [0]
+    row = np.zeros(6, np.int64)
+    with sssp.Graph(row, np.zeros(0, np.uint32), np.zeros(0, np.float32)) as G:
+        G.reorder()
+        d = G.sssp(3, 1.0)
+        assert d[3] == 0 and np.isinf(np.delete(d, 3)).all()
+
+
+def test_self_loops_multi_edges_zero_weights(sssp):
+    rng = np.random.default_rng(7)
+    for trial in range(20):
+        V = int(rng.integers(2, 40))
+        arcs = []
+        for _ in range(int(rng.integers(0, 150))):
+            u, v = int(rng.integers(V)), int(rng.integers(V))
+            arcs.append((u, v, int(rng.integers(0, 5))))
+        row, col, w = csr_from_arcs(V, arcs)
+        s = int(rng.integers(V))
+        exp = oracle.dijkstra(row, col, w, s)
+        with sssp.Graph(row, col, w) as G:
+            if trial % 2:
+                G.reorder()
+            for d in (1, 3, 1e9):
+                assert_same(G.sssp(s, d), exp, f"trial {trial} delta {d}")
+
+
+def test_hub_chunks(sssp):
+    """A star with 20000 leaves plus a ring: light and heavy ranges > 4096 arcs."""
+    n = 20000
+    rng = np.random.default_rng(3)
+    arcs = []
+    for i in range(1, n + 1):
+        w = int(rng.integers(1, 100))
+        arcs += [(0, i, w), (i, 0, w)]
+        j = i % n + 1
+        arcs += [(i, j, 3), (j, i, 3)]
+    row, col, w = csr_from_arcs(n + 1, arcs)
+    for s in (0, 17):
+        exp = oracle.dijkstra(row, col, w, s)
+        with sssp.Graph(row, col, w) as G:
+            G.reorder()
+            for d in (10, 60):
+                assert_same(G.sssp(s, d), exp, f"hub src={s} delta={d}")
+                assert G.stats()["hub_chunks"] > 0
+
+
+def test_forced_overflow_rescans(sssp):
+    """Tiny queues and ring force the dropped-push -> rescan fall-back."""
+    g = gen.kronecker(14, 16, seed=9)
+    s = int(gen.sample_sources(g, 1, seed=2)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_SLOT_CAPACITY, 4096)
+        assert_same(G.sssp(s, 64), exp, "slot capacity 4096")
+        assert G.stats()["rescans"] > 0
+        G.set_param(sssp.SSSP_PARAM_SLOT_CAPACITY, 0)
+        G.set_param(sssp.SSSP_PARAM_RING_SLOTS, 4)
+        assert_same(G.sssp(s, 4), exp, "ring 4, delta 4")
+        assert G.stats()["rescans"] > 0
+
+
+@pytest.mark.parametrize("param,value", [(1, 1), (3, 1), (3, 17)])
+def test_launch_shapes(sssp, param, value):
+    g = gen.kronecker(12, 16, seed=4)
+    s = int(gen.sample_sources(g, 1, seed=5)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.set_param(param, value)
+        assert_same(G.sssp(s, 32), exp, f"param {param}={value}")
+
+
+def test_determinism_repeated(sssp):
+    g = gen.kronecker(12, 16, seed=6)
+    s = int(gen.sample_sources(g, 1, seed=5)[0])
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        first = G.sssp(s, 16).copy()
+        for _ in range(50):
+            assert_same(G.sssp(s, 16), first, "repeat")
+
+
+# ---------------------------------------------------- PRO vs oracle -------
+@pytest.mark.parametrize("wt", ["u32", "f32"])
+def test_pro_matches_oracle(sssp, wt):
+    g = gen.kronecker(12, 16, seed=31, weights=wt)
+    ref = oracle.pro_reorder(g.row, g.col, g.w)
+    delta = 32 if wt == "u32" else 0.25
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        ex = G.export_csr(delta)
+    assert np.array_equal(ex["new2old"], ref["new2old"])
+    assert np.array_equal(ex["adj"], ref["adj"])
+    assert np.array_equal(bits(ex["val"]), bits(ref["val"]))
+    assert np.array_equal(ex["rowlist"], oracle.pro_rowlist(ref["row"], ref["val"], delta))
+
+
+# ------------------------------------------------------------- stats ------
+def test_stats_invariants(sssp):
+    g = gen.kronecker(13, 16, seed=8)
+    s = int(gen.sample_sources(g, 1, seed=1)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    reach = int((exp != INF).sum())
+    ref = oracle.pro_reorder(g.row, g.col, g.w)
+    rl = oracle.pro_rowlist(ref["row"], ref["val"], 32)
+    heavy_deg = rl[2::2] - rl[1::2]  # end - heavy per new vertex
+    reach_new = exp[ref["new2old"]] != INF
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.sssp(s, 32)
+        st = G.stats()
+    assert st["reachable"] == reach
+    # valid updates = reachable - 1; every update is >= valid
+    assert st["updates"] >= reach - 1
+    # each reachable vertex's heavy arcs are relaxed exactly once (u32 weights)
+    assert st["heavy_vertices"] == reach
+    assert st["heavy_arcs"] == int(heavy_deg[reach_new].sum())
+    assert st["vertices_settled"] >= reach
+
+
+# ---------------------------------------------------------- ABI errors ----
+def test_abi_errors_on_device(sssp):
+    g = gen.kronecker(8, 8, seed=1)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances()
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+        for bad in (0, -1, float("nan")):
+            with pytest.raises(sssp.SSSPError) as e:
+                G.run(0, bad)
+            assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+        for src in (-1, g.V):
+            with pytest.raises(sssp.SSSPError):
+                G.run(src, 4)
+        G.run(int(gen.sample_sources(g, 1)[0]), 4)
+        G.distances()
+        G.reorder()
+        G.reorder()  # idempotent
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances()  # reorder invalidates the result
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+    bad_col = g.col.copy()
+    bad_col[5] = g.V
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph(g.row, bad_col, g.w)
+    assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+    bad_row = g.row.copy()
+    bad_row[3], bad_row[4] = bad_row[4], bad_row[3] - 1
+    with pytest.raises(sssp.SSSPError):
+        sssp.Graph(bad_row, g.col, g.w)
+    for x in (-1.0, float("nan"), float("inf")):
+        wf = g.w.astype(np.float32)
+        wf[2] = x
+        with pytest.raises(sssp.SSSPError):
+            sssp.Graph(g.row, g.col, wf)
+
+
+def test_u32_overflow_reported(sssp):
+    row, col, w = csr_from_arcs(3, [(0, 1, 0xFFFFFFF0), (1, 2, 0x20)])
+    with sssp.Graph(row, col, w) as G:
+        G.run(0, 1e9)
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances()
+        assert e.value.status == sssp.SSSP_ERR_OVERFLOW
+
+
+def test_negative_zero_weight_canonicalised(sssp):
+    row, col, w = csr_from_arcs(3, [(0, 1, np.float32(-0.0)), (1, 2, np.float32(0.5))], np.float32)
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        d = G.sssp(0, 0.25)
+    assert bits(d).tolist() == bits(np.array([0, 0, 0.5], np.float32)).tolist()
+
+
+# --------------------------------------------------- device memory path ---
+def test_device_inputs_and_outputs(sssp):
+    import torch
+
+    g = gen.kronecker(11, 16, seed=12)
+    s = int(gen.sample_sources(g, 1, seed=1)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    row = torch.from_numpy(g.row).cuda()
+    col = torch.from_numpy(g.col.view(np.int32)).cuda()
+    w = torch.from_numpy(g.w.view(np.int32)).cuda()
+    stream = torch.cuda.Stream()
+    with sssp.Graph(row, col, w, stream=stream) as G:
+        G.reorder()
+        out = torch.empty(g.V, dtype=torch.int32, device="cuda")
+        G.run(s, 32)
+        G.distances(out)
+        torch.cuda.synchronize()
+        assert_same(out.cpu().numpy().view(np.uint32), exp, "device out")
+        # batch into a device matrix
+        srcs = gen.sample_sources(g, 4, seed=9)
+        mat = torch.empty((4, g.V), dtype=torch.int32, device="cuda")
+        G.run_batch(srcs, 32, mat)
+        torch.cuda.synchronize()
+        for i, ss in enumerate(srcs):
+            assert_same(mat[i].cpu().numpy().view(np.uint32), oracle.dijkstra(g.row, g.col, g.w, int(ss)), "batch")
