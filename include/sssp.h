@@ -161,6 +161,21 @@ sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
  * reset != 0 zeroes the accumulators after reporting. */
 sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_t* launches, int reset);
 
+/* Scheduler timeline of the last run: one entry per grid barrier (written by
+ * the last CTA to arrive, before it releases the others) plus a kernel-start
+ * entry (which = 99). which: 0 end of phase 1, 1 end of phases 2&3, 2/3
+ * rescan stages, 4/5 sweep fall-back stages. Up to 4096 entries. */
+typedef struct sssp_trace_entry {
+    uint64_t t_ns;   /* %globaltimer */
+    uint32_t which;  /* barrier kind (see above) */
+    uint32_t cur;    /* current bucket after the scheduler step */
+    uint32_t tail;   /* entries in that bucket's queue */
+    uint32_t mode;   /* next mode: 0 phase 1, 1 phase 2, 2 done, 3/4 rescan, 5/6 sweep */
+    uint32_t far_min, pad;
+} sssp_trace_entry;
+sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
+                           int64_t* n_entries);
+
 /* Library/device info: number of SMs of the handle's device. */
 int sssp_device_sm_count(sssp_graph_t g);
 

@@ -17,7 +17,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsssp.so")
+LIB_PATH = os.environ.get("SSSP_LIB") or os.path.join(_HERE, "libsssp.so")  # override: experiments only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libsssp.so not built at {LIB_PATH}; run __graft_entry__.build() (no CPU fallback exists)")
@@ -49,7 +49,7 @@ EXPORTS = (
     "sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
-    "sssp_kernel_time",
+    "sssp_kernel_time", "sssp_get_trace",
 )
 
 
@@ -84,6 +84,16 @@ _lib.sssp_set_param.argtypes = [_P, _I, _I64]
 _lib.sssp_device_sm_count.argtypes = [_P]
 _lib.sssp_kernel_time.argtypes = [_P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64), _I]
 _lib.sssp_kernel_time.restype = _I
+
+
+class sssp_trace_entry(ctypes.Structure):
+    _fields_ = [("t_ns", ctypes.c_uint64), ("which", ctypes.c_uint32), ("cur", ctypes.c_uint32),
+                ("tail", ctypes.c_uint32), ("mode", ctypes.c_uint32), ("far_min", ctypes.c_uint32),
+                ("pad", ctypes.c_uint32)]
+
+
+_lib.sssp_get_trace.argtypes = [_P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]
+_lib.sssp_get_trace.restype = _I
 for _n in ("sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
            "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param"):
     getattr(_lib, _n).restype = _I
@@ -207,6 +217,20 @@ def sssp_kernel_time(h, reset=False):
     return t.value, n.value
 
 
+def sssp_get_trace(h, max_entries=4096):
+    """Barrier timeline of the last run: list of dicts (t_us relative to kernel start)."""
+    buf = (sssp_trace_entry * max_entries)()
+    n = ctypes.c_int64()
+    _check(_lib.sssp_get_trace(h, buf, max_entries, ctypes.byref(n)), "sssp_get_trace")
+    out = []
+    t0 = buf[0].t_ns if n.value else 0
+    for i in range(min(n.value, max_entries)):
+        e = buf[i]
+        out.append(dict(t_us=(e.t_ns - t0) / 1e3, which=e.which, cur=e.cur, tail=e.tail, mode=e.mode,
+                        far_min=e.far_min))
+    return out
+
+
 def sssp_device_sm_count(h):
     return int(_lib.sssp_device_sm_count(h))
 
@@ -269,6 +293,9 @@ class Graph:
 
     def kernel_time(self, reset=False):
         return sssp_kernel_time(self.h, reset)
+
+    def trace(self):
+        return sssp_get_trace(self.h)
 
     def set_stream(self, stream):
         sssp_set_stream(self.h, stream)

@@ -13,7 +13,15 @@ typedef int64_t i64;
 
 // ---- loads / stores with explicit cache behaviour --------------------------
 // Arcs are streamed (read ~once per SSSP): evict-first in L1/L2.
-__device__ __forceinline__ uint2 ld_stream_u2(const uint2* p) { return __ldcs(p); }
+__device__ __forceinline__ uint2 ld_stream_u2(const uint2* p) {
+  uint2 v;
+  u64 pol;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
+      : "=r"(v.x), "=r"(v.y)
+      : "l"(p), "l"(pol));
+  return v;
+}
 // Coherent (L2) load of mutable data (dist[], queue words).
 __device__ __forceinline__ u32 ld_cg(const u32* p) { return __ldcg(p); }
 __device__ __forceinline__ u64 ld_relaxed_u64(const u64* p) {

@@ -9,7 +9,7 @@
 //     ranges staged in shared memory), 32 <= l < 256 -> warp per vertex,
 //     256 <= l <= 4096 -> CTA per vertex, l > 4096 -> ceil(l/4096) chunks any
 //     CTA may claim (reading R11). Improved vertices are pushed
-//     into the near queue (same bucket: visible at once, no level barrier,
+//     into the near queue (same bucket: visible without a level barrier,
 //     P:1100-1103) or a far bucket queue. The phase ends at quiescence:
 //     pend (pushed - completed) == 0 (manager/worker end rule).
 //   phases 2&3 (Alg. 2 l.13-19): after a grid barrier, heavy arcs
@@ -19,23 +19,37 @@
 //
 // Data (all device memory): dist[V] u32 (f32 as IEEE bits: order-preserving
 // for w >= 0, so one atomicMin.u32 serves both weight types, Alg. 1 l.3);
-// a ring of K bucket queues of packed u64 entries (d << 32 | v), each with one
-// 64-bit word (tail << 32 | pend) so a single atomicAdd both reserves slots and
-// counts pending work; entries are published by value (SENTINEL = empty).
+// a ring of K bucket queues of packed u64 entries (d << 32 | v). Each queue
+// has its own 128-byte control line: word = (tail << 32 | pend), so one
+// atomicAdd both reserves entries and counts pending work, and head, the
+// consumers' ticket counter. Consumers claim position ranges with atomicAdd
+// (never fails; a range may run ahead of tail and is filled as producers
+// publish); entries are published by value (SENTINEL = empty). Producers
+// stage pushes per warp in shared memory (one global reservation per flush).
 // Pushes beyond the ring horizon or beyond a queue's capacity are dropped and
 // recorded in far_min; the scheduler then rebuilds the ring from dist[]
-// (topological rescan, as the paper's phase 3 loops over all V, Alg. 2 l.13).
+// (topological rescan, as the paper's phase 3 loops over all V, Alg. 2 l.13)
+// or, for the current bucket, finishes it with Bellman-Ford sweeps.
 #pragma once
 #include "common.cuh"
 
 namespace sssp {
 
+#ifndef SSSP_MINB
+#define SSSP_MINB 4  // persistent CTAs per SM the register budget is sized for
+#endif
 constexpr int DS_THREADS = 256;
 constexpr int DS_WARPS = DS_THREADS / 32;
 constexpr u32 BIN_WARP = 32;     // beta
 constexpr u32 BIN_CTA = 256;     // alpha
 constexpr u32 HUB_CHUNK = 4096;
-constexpr int UNROLL = 4;
+#ifndef SSSP_UNROLL
+#define SSSP_UNROLL 4
+#endif
+#ifndef SSSP_PROBE_L1
+#define SSSP_PROBE_L1 1  // dist probes through L1 (a stale value is a safe filter)
+#endif
+constexpr int UNROLL = SSSP_UNROLL;
 constexpr u64 SENTINEL = ~0ULL;
 constexpr u32 NONE = 0xFFFFFFFFu;
 constexpr u32 CHUNK_FLAG = 0x80000000u;
@@ -67,14 +81,41 @@ enum {
   ST_N
 };
 
-struct Ctl {
-  u32 cur, lim, mode, far_min;
-  u32 p2_begin, p2_end, p2_head, err;
-  u32 bar_count, bar_gen, epochs, rescans;
-  u32 rescan_base, changed, sweep_first, sweeps;
-  u64 hub_word;
-  u32 hub_head, pad3;
+struct __align__(128) SlotCtl {
+  u64 word;  // (tail << 32) | pend
+  u32 head;  // consumer tickets
+  u32 p2;    // prefix already handled by phase 2
+  u32 pad[28];
 };
+
+struct __align__(128) Ctl {
+  u32 cur, lim, mode, far_min;
+  u32 p2_begin, p2_end, err, epochs;
+  u32 rescans, rescan_base, changed, sweep_first;
+  u32 sweeps, trace_n, pad1, pad2;
+  u32 pad_a[16];
+  u32 bar_count, pad3[31];   // own line: arrivals
+  u32 bar_gen, pad4[31];     // own line: spun on
+  u32 p2_head, pad5[31];     // own line: phase-2 static tickets
+  u64 hub_word;              // phase-2 chunk queue: (tail << 32) | pend
+  u32 hub_head, pad6[29];
+};
+
+constexpr u32 TRACE_CAP = 4096;
+struct TraceEnt {
+  u64 t_ns;   // %globaltimer when the last CTA arrived
+  u32 which;  // SYNC_* (99 = kernel start)
+  u32 cur;    // current bucket
+  u32 tail;   // entries in the current bucket's queue
+  u32 mode;   // mode chosen by the scheduler
+  u32 far_min, pad;
+};
+
+__device__ __forceinline__ u64 globaltimer() {
+  u64 t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 struct Params {
   const longlong2* rowp;  // [V+1] {start, heavy}
@@ -82,12 +123,11 @@ struct Params {
   u32* dist;              // [V]
   u32* xd;                // [V] sweep fall-back: distance at last light expansion
   Ctl* ctl;
-  u64* word;              // [K]
-  u32* head;              // [K]
-  u32* p2;                // [K]
+  SlotCtl* sc;            // [K]
   u64* items;             // [K * cap]
   u64* hub_items;         // [hub_cap]
   unsigned long long* stats;  // [ST_N]
+  TraceEnt* trace;            // [TRACE_CAP] barrier timeline of the last run
   u32 V, K, kmask, cap, hub_cap;
   u32 delta_u;       // u32 graphs: integer Delta >= 1
   float inv_delta;   // f32 graphs: fl32(1/Delta)
@@ -95,25 +135,48 @@ struct Params {
   u32 claim_max;
 };
 
+constexpr u32 TASK = 32 * UNROLL;  // arcs per warp task
+constexpr u32 PB_CAP = 256;        // staged pushes per warp (>= 32 * UNROLL)
+
 struct Smem {
-  u64 items[DS_THREADS];
-  i64 wl_beg[DS_THREADS];
-  u32 wl_len[DS_THREADS];
-  u32 wl_d[DS_THREADS];
-  i64 cl_beg[DS_THREADS];
-  u32 cl_len[DS_THREADS];
-  u32 cl_d[DS_THREADS];
-  i64 sb_beg[DS_WARPS][32];
+  // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
+  // thread bin (small vertices, arcs spread by a warp prefix sum); tasks
+  // [S, S+R): 128-arc slices of the range list (warp-bin vertices, CTA-bin
+  // vertices and hub chunks: a 256..4096-arc vertex is spread over the CTA's
+  // 8 warps = "CTA per vertex"; a 32..255-arc one takes 1-2 tasks = "warp per
+  // vertex"). Any warp may run any task, so warps stay balanced.
+  u32 rl_beg[DS_THREADS];
+  u32 rl_len[DS_THREADS];
+  u32 rl_d[DS_THREADS];
+  u32 rl_toff[DS_THREADS + 1];
+  u32 sb_beg[DS_WARPS][32];
   u32 sb_off[DS_WARPS][32];
   u32 sb_d[DS_WARPS][32];
+  u32 sb_total[DS_WARPS];
+  u32 scan_ws[DS_WARPS];
+  u32 rl_n, rl_tasks, task_next;
+  u64 pb[DS_WARPS][PB_CAP];  // staged pushes (d << 32 | v), bucket resolved at flush
+  u32 pb_n[DS_WARPS];
   unsigned long long st[ST_N];
-  u32 wl_n, wl_next, cl_n;
   u32 claim_h, claim_n, claim_src;
   // control snapshot
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first;
 };
 
 // ---------------------------------------------------------------- helpers --
+// Filter probe of dist[] before the atomicMin (Alg. 1 l.2). Any value ever
+// stored in dist[v] is >= its current value, so a stale (L1-cached) read can
+// only cause an extra atomic, never a missed improvement.
+__device__ __forceinline__ u32 ld_probe(const u32* p) {
+#if SSSP_PROBE_L1
+  u32 v;
+  asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#else
+  return __ldcg(p);
+#endif
+}
+
 template <bool F32>
 __device__ __forceinline__ u32 relax_add(u32 d, u32 w, u32* err) {
   if (F32) {
@@ -143,44 +206,73 @@ __device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
   if (lane_id() == 0 && s) atomicAdd(&sm.st[k], (unsigned long long)s);
 }
 
-// Push (v, nd) into the queue of bucket(nd). Must be called by all 32 lanes.
-// nearb != NONE (sweep fall-back): improvements landing in bucket nearb are
-// not queued; they mark v for the next sweep instead.
+// Publish warp w's staged pushes: per 32 entries, one global reservation per
+// distinct bucket queue (tail and pend in one atomicAdd). Entries beyond the
+// ring horizon or a full queue are dropped and recorded in far_min. In the
+// sweep fall-back (nearb != NONE) entries of bucket nearb mark xd[] instead.
 template <bool F32>
-__device__ __forceinline__ void warp_push(const Params& p, Smem& sm, u32 lim, bool want, u32 v,
-                                          u32 nd, u32 nearb) {
-  const u32 any = __ballot_sync(SSSP_FULL_MASK, want);
-  if (!any) return;
-  if (lane_id() == (u32)(__ffs(any) - 1)) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)__popc(any));
-  u32 x = 0;
-  bool ok = false;
-  if (want) {
-    x = bucket_of<F32>(p, nd);
-    if (x == nearb) {
+__device__ __noinline__ void pb_flush(const Params p, Smem& sm, u32 lim, u32 nearb) {
+  const u32 lane = lane_id(), w = threadIdx.x >> 5;
+  const u32 n = sm.pb_n[w];
+  if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)n);
+  for (u32 i0 = 0; i0 < n; i0 += 32) {
+    const u32 i = i0 + lane;
+    bool ok = i < n;
+    const u64 e = ok ? sm.pb[w][i] : 0ULL;
+    const u32 v = (u32)e, nd = (u32)(e >> 32);
+    const u32 x = ok ? bucket_of<F32>(p, nd) : 0u;
+    if (ok && x == nearb) {
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
-    } else {
-      ok = x <= lim;
-      if (!ok) atomicMin(&p.ctl->far_min, x);  // beyond the ring horizon: rescan later
+      ok = false;
     }
-  }
-  const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
-  if (ok) {
-    const u32 s = x & p.kmask;
-    const u32 peers = __match_any_sync(m, s);
-    const u32 leader = __ffs(peers) - 1;
-    const u32 cnt = __popc(peers);
-    u64 old = 0;
-    if (lane_id() == leader) old = atomicAdd(p.word + s, ((u64)cnt << 32) | cnt);
-    old = __shfl_sync(peers, old, leader);
-    const u32 idx = (u32)(old >> 32) + __popc(peers & lanemask_lt());
-    if (idx < p.cap) {
-      st_relaxed_u64(p.items + (u64)s * p.cap + idx, ((u64)nd << 32) | v);
-    } else {  // queue full: undo the pending count, recover by rescan
-      atomicAdd(p.word + s, ~0ULL);
+    if (ok && x > lim) {  // beyond the ring horizon: rescan later
       atomicMin(&p.ctl->far_min, x);
+      ok = false;
+    }
+    const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
+    if (ok) {
+      const u32 s = x & p.kmask;
+      const u32 peers = __match_any_sync(m, s);
+      const u32 leader = __ffs(peers) - 1;
+      const u32 cnt = __popc(peers);
+      u64 old = 0;
+      if (lane == leader) old = atomicAdd(&p.sc[s].word, ((u64)cnt << 32) | cnt);
+      old = __shfl_sync(peers, old, leader);
+      const u32 idx = (u32)(old >> 32) + __popc(peers & lanemask_lt());
+      if (idx < p.cap) {
+        st_relaxed_u64(p.items + (u64)s * p.cap + idx, e);
+      } else {  // queue full: undo the pending count, recover later
+        atomicAdd(&p.sc[s].word, ~0ULL);
+        atomicMin(&p.ctl->far_min, x);
+      }
     }
   }
+  __syncwarp();
+  if (lane == 0) sm.pb_n[w] = 0;
+  __syncwarp();
+}
+
+// Stage up to UNROLL pushes per lane into the warp's buffer (all 32 lanes).
+template <bool F32>
+__device__ __forceinline__ void stage_pushes(const Params& p, Smem& sm, u32 lim, u32 nearb,
+                                             const bool (&want)[UNROLL], const u32 (&v)[UNROLL],
+                                             const u32 (&nd)[UNROLL]) {
+  u32 c = 0;
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) c += want[k];
+  if (!__any_sync(SSSP_FULL_MASK, c != 0)) return;
+  const u32 w = threadIdx.x >> 5;
+  u32 tot;
+  const u32 off = warp_exclusive_scan(c, &tot);
+  if (sm.pb_n[w] + tot > PB_CAP) pb_flush<F32>(p, sm, lim, nearb);
+  u32 pos = sm.pb_n[w] + off;
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k)
+    if (want[k]) sm.pb[w][pos++] = ((u64)nd[k] << 32) | v[k];
+  __syncwarp();
+  if (lane_id() == 0) sm.pb_n[w] += tot;
+  __syncwarp();
 }
 
 // Relax UNROLL arcs per thread (independent loads in flight: arcs, then dist
@@ -188,7 +280,7 @@ __device__ __forceinline__ void warp_push(const Params& p, Smem& sm, u32 lim, bo
 // light/heavy split is a per-arc predicate (the divergence PRO removes).
 template <bool F32, bool PRO, int PH>
 __device__ __forceinline__ void relax_group(const Params& p, Smem& sm, u32 lim, u32 nearb,
-                                            const i64 (&idx)[UNROLL], const bool (&valid)[UNROLL],
+                                            const u32 (&idx)[UNROLL], const bool (&valid)[UNROLL],
                                             const u32 (&d)[UNROLL]) {
   uint2 a[UNROLL];
   u32 nd[UNROLL];
@@ -202,15 +294,17 @@ __device__ __forceinline__ void relax_group(const Params& p, Smem& sm, u32 lim, 
     if (!PRO) take = take && ((PH == 1) ? (a[k].y < p.delta_bits) : (a[k].y >= p.delta_bits));
     want[k] = take;
     nd[k] = take ? relax_add<F32>(d[k], a[k].y, &p.ctl->err) : NONE;
-    cur[k] = take ? ld_cg(p.dist + a[k].x) : 0u;
+    cur[k] = take ? ld_probe(p.dist + a[k].x) : 0u;
   }
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     want[k] = want[k] && nd[k] < cur[k];  // check before the atomic (Alg. 1 l.2)
     if (want[k]) want[k] = nd[k] < atomicMin(p.dist + a[k].x, nd[k]);  // Alg. 1 l.3
   }
+  u32 vv[UNROLL];
 #pragma unroll
-  for (int k = 0; k < UNROLL; ++k) warp_push<F32>(p, sm, lim, want[k], a[k].x, nd[k], nearb);
+  for (int k = 0; k < UNROLL; ++k) vv[k] = a[k].x;
+  stage_pushes<F32>(p, sm, lim, nearb, want, vv, nd);
 }
 
 // Range of an item for phase PH: PRO -> light [start, heavy) / heavy [heavy, end);
@@ -228,44 +322,39 @@ __device__ __forceinline__ void item_range(const Params& p, u32 v, i64& b, i64& 
 }
 
 // ------------------------------------------------------------ batch -------
-// Process the CTA's claimed items (one per thread; has = thread holds one).
+// Process the CTA's claimed items (at most one per thread; has = holds one).
 // src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
 // phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
-// into the current bucket, hubs stay in the CTA bin).
+// into the current bucket, hubs stay in the range list).
 template <bool F32, bool PRO, int PH>
-__device__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 lim, u32 src,
-                              u32 slot) {
+__device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 lim,
+                                              u32 src, u32 slot) {
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const bool sweep = src == SRC_SWEEP;
   const u32 nearb = sweep ? sm.cur : NONE;
-  bool small = false;
-  i64 beg = 0;
-  u32 len = 0, d = 0;
-  u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0;
+  bool small = false, listed = false;
+  u32 beg = 0, len = 0, d = 0;
+  u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0;
   if (has) {
     const u32 lo = (u32)it, hi = (u32)(it >> 32);
-    bool is_chunk = (lo & CHUNK_FLAG) != 0;
+    const bool is_chunk = (lo & CHUNK_FLAG) != 0;
     const u32 v = lo & ~CHUNK_FLAG;
-    bool live = false;
     if (is_chunk) {
       // Chunk items in the phase-2 static range are phase-1 work already done.
-      live = !(PH == 2 && src == SRC_STATIC);
-      if (live) {
+      if (!(PH == 2 && src == SRC_STATIC)) {
         i64 rb, re;
         item_range<PRO, PH>(p, v, rb, re);
-        beg = rb + (i64)hi * HUB_CHUNK;
-        len = (u32)min((i64)HUB_CHUNK, re - beg);
+        const i64 b = rb + (i64)hi * HUB_CHUNK;
+        beg = (u32)b;
+        len = (u32)min((i64)HUB_CHUNK, re - b);
         d = ld_cg(p.dist + v);  // current distance: a valid path length (<= spawning d)
         c_arcs = len;
-        u32 i = atomicAdd(&sm.cl_n, 1u);
-        sm.cl_beg[i] = beg;
-        sm.cl_len[i] = len;
-        sm.cl_d[i] = d;
+        listed = true;
       }
     } else {
       const u32 cd = ld_cg(p.dist + v);
       d = hi;
-      live = (PH == 1) ? (d <= cd) : (d == cd);  // stale filter / settled-final filter
+      const bool live = (PH == 1) ? (d <= cd) : (d == cd);  // stale / settled-final filter
       if (!live) {
         c_stale = (PH == 1);
       } else {
@@ -273,12 +362,12 @@ __device__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 l
         i64 rb, re;
         item_range<PRO, PH>(p, v, rb, re);
         const i64 l = re - rb;
-        c_arcs = (u32)min(l, (i64)0xFFFFFFFF);
+        c_arcs = (u32)l;
         if (l > (i64)HUB_CHUNK && !sweep) {  // hub: ceil(l/4096) chunks any CTA may claim
           const u32 nc = (u32)((l + HUB_CHUNK - 1) / HUB_CHUNK);
           c_chunks = nc;
           c_arcs = 0;  // counted when the chunks run
-          u64* word = (PH == 1) ? p.word + slot : &p.ctl->hub_word;
+          u64* word = (PH == 1) ? &p.sc[slot].word : &p.ctl->hub_word;
           u64* q = (PH == 1) ? p.items + (u64)slot * p.cap : p.hub_items;
           const u32 qcap = (PH == 1) ? p.cap : p.hub_cap;
           const u32 base = (u32)(atomicAdd(word, ((u64)nc << 32) | nc) >> 32);
@@ -288,24 +377,20 @@ __device__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 l
             } else {
               atomicAdd(word, ~0ULL);
               if (PH == 1)
-                atomicMin(&p.ctl->far_min, sm.cur);  // lost phase-1 work: rescan this bucket
+                atomicMin(&p.ctl->far_min, sm.cur);  // lost phase-1 work: sweep this bucket
               else
                 atomicOr(&p.ctl->err, ERR_INTERNAL);
             }
           }
-        } else if (l >= (i64)BIN_CTA) {
-          u32 i = atomicAdd(&sm.cl_n, 1u);
-          sm.cl_beg[i] = rb;
-          sm.cl_len[i] = (u32)l;
-          sm.cl_d[i] = d;
         } else if (l >= (i64)BIN_WARP) {
-          u32 i = atomicAdd(&sm.wl_n, 1u);
-          sm.wl_beg[i] = rb;
-          sm.wl_len[i] = (u32)l;
-          sm.wl_d[i] = d;
+          beg = (u32)rb;
+          len = (u32)l;
+          listed = true;
+          c_c = l >= (i64)BIN_CTA;
+          c_w = !c_c;
         } else if (l > 0) {
           small = true;
-          beg = rb;
+          beg = (u32)rb;
           len = (u32)l;
         }
       }
@@ -317,112 +402,128 @@ __device__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 l
   st_add(sm, PH == 1 ? ST_LIGHT : ST_HEAVY, c_arcs);
   st_add(sm, ST_CHUNKS, c_chunks);
   st_add(sm, ST_BIN_T, small ? 1u : 0u);
+  st_add(sm, ST_BIN_W, c_w);
+  st_add(sm, ST_BIN_C, c_c);
 
-  // ---- thread bin: a warp's small vertices, arcs spread by a warp prefix sum
+  // ---- stage: thread bin (warp prefix sum) and range list (block scan)
   {
-    u32 total;
-    const u32 off = warp_exclusive_scan(small ? len : 0u, &total);
-    if (total) {
-      sm.sb_beg[w][lane] = beg;
-      sm.sb_off[w][lane] = off;
-      sm.sb_d[w][lane] = d;
-      __syncwarp();
-      for (u32 j0 = 0; j0 < total; j0 += 32 * UNROLL) {
-        i64 idx[UNROLL];
-        bool valid[UNROLL];
-        u32 dd[UNROLL];
+    u32 stot;
+    const u32 soff = warp_exclusive_scan(small ? len : 0u, &stot);
+    sm.sb_beg[w][lane] = beg;
+    sm.sb_off[w][lane] = soff;  // monotone; zero-length lanes never own an arc
+    sm.sb_d[w][lane] = d;
+    const u32 x = listed ? ((1u << 16) | ((len + TASK - 1) / TASK)) : 0u;
+    u32 wt;
+    const u32 ex = warp_exclusive_scan(x, &wt);
+    if (lane == 31) {
+      sm.scan_ws[w] = wt;
+      sm.sb_total[w] = stot;
+    }
+    __syncthreads();
+    u32 acc = 0, tot = 0;
 #pragma unroll
-        for (int k = 0; k < UNROLL; ++k) {
-          const u32 j = j0 + k * 32 + lane;
-          valid[k] = j < total;
-          u32 o = 0;  // owner: last lane with sb_off <= j
-#pragma unroll
-          for (u32 step = 16; step; step >>= 1)
-            if (sm.sb_off[w][o + step] <= j) o += step;
-          idx[k] = sm.sb_beg[w][o] + (j - sm.sb_off[w][o]);
-          dd[k] = sm.sb_d[w][o];
-        }
-        relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
-      }
-      __syncwarp();
+    for (int i = 0; i < DS_WARPS; ++i) {
+      const u32 s = sm.scan_ws[i];
+      if (i < (int)w) acc += s;
+      tot += s;
+    }
+    const u32 off = ex + acc;
+    if (listed) {
+      const u32 i = off >> 16;
+      sm.rl_beg[i] = beg;
+      sm.rl_len[i] = len;
+      sm.rl_d[i] = d;
+      sm.rl_toff[i] = off & 0xFFFFu;
+    }
+    if (tid == 0) {
+      sm.rl_n = tot >> 16;
+      sm.rl_tasks = tot & 0xFFFFu;
+      sm.rl_toff[tot >> 16] = tot & 0xFFFFu;
+      sm.task_next = 0;
     }
   }
-  __syncthreads();
-  // ---- warp bin: one warp per vertex (32 <= l < 256)
-  if (tid == 0) {
-    sm.st[ST_BIN_W] += sm.wl_n;
-    sm.st[ST_BIN_C] += sm.cl_n;
-  }
+  __syncthreads();  // task pool complete
+
+  // small-task offsets per warp
+  u32 soff_w[DS_WARPS + 1];
+  soff_w[0] = 0;
+#pragma unroll
+  for (int i = 0; i < DS_WARPS; ++i) soff_w[i + 1] = soff_w[i] + (sm.sb_total[i] + TASK - 1) / TASK;
+  const u32 S = soff_w[DS_WARPS];
+  const u32 ntask = S + sm.rl_tasks, nl = sm.rl_n;
   for (;;) {
-    u32 i = 0;
-    if (lane == 0) i = atomicAdd(&sm.wl_next, 1u);
-    i = __shfl_sync(SSSP_FULL_MASK, i, 0);
-    if (i >= sm.wl_n) break;
-    const i64 b = sm.wl_beg[i];
-    const u32 l = sm.wl_len[i];
-    const u32 dv = sm.wl_d[i];
-    for (u32 j0 = 0; j0 < l; j0 += 32 * UNROLL) {
-      i64 idx[UNROLL];
-      bool valid[UNROLL];
-      u32 dd[UNROLL];
+    u32 t = 0;
+    if (lane == 0) t = atomicAdd(&sm.task_next, 1u);
+    t = __shfl_sync(SSSP_FULL_MASK, t, 0);
+    if (t >= ntask) break;
+    u32 idx[UNROLL];
+    bool valid[UNROLL];
+    u32 dd[UNROLL];
+    if (t < S) {  // thread-bin slice of warp ww
+      u32 ww = 0;
+#pragma unroll
+      for (int i = 1; i < DS_WARPS; ++i) ww += (t >= soff_w[i]);
+      const u32 j0 = (t - soff_w[ww]) * TASK, total = sm.sb_total[ww];
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
         const u32 j = j0 + k * 32 + lane;
-        valid[k] = j < l;
-        idx[k] = b + j;
-        dd[k] = dv;
+        valid[k] = j < total;
+        u32 o = 0;  // owner: last lane with sb_off <= j
+#pragma unroll
+        for (u32 step = 16; step; step >>= 1)
+          if (sm.sb_off[ww][o + step] <= j) o += step;
+        idx[k] = sm.sb_beg[ww][o] + (j - sm.sb_off[ww][o]);
+        dd[k] = sm.sb_d[ww][o];
       }
-      relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
-    }
-  }
-  // ---- CTA bin: the whole CTA per vertex / chunk (256 <= l <= 4096)
-  const u32 ncl = sm.cl_n;
-  for (u32 i = 0; i < ncl; ++i) {
-    const i64 b = sm.cl_beg[i];
-    const u32 l = sm.cl_len[i];
-    const u32 dv = sm.cl_d[i];
-    for (u32 j0 = 0; j0 < l; j0 += DS_THREADS * UNROLL) {
-      i64 idx[UNROLL];
-      bool valid[UNROLL];
-      u32 dd[UNROLL];
+    } else {  // range-list slice
+      const u32 tr = t - S;
+      u32 lo = 0, hi = nl;  // entry i with toff[i] <= tr < toff[i+1]
+      while (hi - lo > 1) {
+        const u32 mid = (lo + hi) >> 1;
+        if (sm.rl_toff[mid] <= tr)
+          lo = mid;
+        else
+          hi = mid;
+      }
+      const u32 sub = (tr - sm.rl_toff[lo]) * TASK;
+      const u32 b = sm.rl_beg[lo] + sub;
+      const u32 l = sm.rl_len[lo] - sub;
+      const u32 dv = sm.rl_d[lo];
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
-        const u32 j = j0 + k * DS_THREADS + tid;
+        const u32 j = k * 32 + lane;
         valid[k] = j < l;
         idx[k] = b + j;
         dd[k] = dv;
       }
-      relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
     }
+    relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
   }
+  if (sm.pb_n[w]) pb_flush<F32>(p, sm, lim, nearb);  // publish before reporting completion
   __syncthreads();
-  if (tid == 0) {
-    sm.wl_n = 0;
-    sm.wl_next = 0;
-    sm.cl_n = 0;
-  }
 }
 
 // --------------------------------------------------------- grid barrier ---
+__device__ __forceinline__ void enter_sweep(volatile Ctl* c) {
+  c->changed = 0;
+  c->sweep_first = 1;
+  c->sweeps = c->sweeps + 1;
+  c->mode = MODE_SWEEP_LIGHT;
+}
+
 // Last CTA to arrive runs the serial scheduler step (fused phase 3).
 __device__ void decide(const Params& p, u32 which) {
   volatile Ctl* c = p.ctl;
-  volatile u64* word = p.word;
-  volatile u32* head = p.head;
-  volatile u32* p2 = p.p2;
+  volatile SlotCtl* sc = p.sc;
   const u32 K = p.K;
   if (which == SYNC_P1) {
     const u32 cur = c->cur, s = cur & p.kmask;
-    if (c->far_min <= cur) {  // phase-1 work was dropped (queue full): sweep fall-back
-      c->changed = 0;
-      c->sweep_first = 1;
-      c->sweeps = c->sweeps + 1;
-      c->mode = MODE_SWEEP_LIGHT;
+    if (c->far_min <= cur) {  // phase-1 work was dropped (queue full)
+      enter_sweep(c);
       return;
     }
-    const u64 wv = word[s];
-    const u32 tail = min((u32)(wv >> 32), p.cap);
-    const u32 b = p2[s];
+    const u32 tail = min((u32)(sc[s].word >> 32), p.cap);
+    const u32 b = sc[s].p2;
     c->p2_begin = b;
     c->p2_end = tail;
     c->p2_head = b;
@@ -431,14 +532,11 @@ __device__ void decide(const Params& p, u32 which) {
     c->mode = MODE_PHASE2;
   } else if (which == SYNC_P2) {
     const u32 cur = c->cur, s = cur & p.kmask;
-    p2[s] = c->p2_end;
+    sc[s].p2 = c->p2_end;
     const u32 fm = c->far_min;
-    if ((u32)word[s] != 0) {  // f32: a heavy relaxation rounded into bucket cur
+    if ((u32)sc[s].word != 0) {  // f32: a heavy relaxation rounded into bucket cur
       if (fm <= cur) {
-        c->changed = 0;
-        c->sweep_first = 1;
-        c->sweeps = c->sweeps + 1;
-        c->mode = MODE_SWEEP_LIGHT;
+        enter_sweep(c);
       } else {
         c->mode = MODE_PHASE1;
         c->epochs = c->epochs + 1;
@@ -447,7 +545,7 @@ __device__ void decide(const Params& p, u32 which) {
     }
     u32 nxt = NONE;
     for (u32 x = cur + 1; x <= c->lim && x != NONE; ++x)
-      if ((u32)(word[x & p.kmask] >> 32) != 0) {
+      if ((u32)(sc[x & p.kmask].word >> 32) != 0) {
         nxt = x;
         break;
       }
@@ -460,19 +558,19 @@ __device__ void decide(const Params& p, u32 which) {
       c->mode = MODE_RESCAN_CLEAR;
       return;
     }
-    word[s] = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
-    head[s] = 0;
-    p2[s] = 0;
-    const u64 lim = (u64)cur + K - 1;  // excludes slot s: it is reset now
+    sc[s].word = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
+    sc[s].head = 0;
+    sc[s].p2 = 0;
+    const u64 lim = (u64)cur + K - 1;  // excludes slot s of bucket cur+K: reset just now
     c->lim = (u32)min(lim, (u64)NONE - 1);
     c->cur = nxt;
     c->mode = MODE_PHASE1;
     c->epochs = c->epochs + 1;
   } else if (which == SYNC_RC) {
     for (u32 s = 0; s < K; ++s) {
-      word[s] = 0;
-      head[s] = 0;
-      p2[s] = 0;
+      sc[s].word = 0;
+      sc[s].head = 0;
+      sc[s].p2 = 0;
     }
     const u32 r = c->rescan_base;
     c->far_min = NONE;
@@ -507,14 +605,29 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
     if (arrived == gridDim.x - 1) {
       c->bar_count = 0;
       __threadfence();
+      const u64 t = globaltimer();
       decide(p, which);
+      volatile Ctl* vc = c;
+      const u32 tn = vc->trace_n;
+      if (tn < TRACE_CAP) {
+        TraceEnt e;
+        e.t_ns = t;
+        e.which = which;
+        e.cur = vc->cur;
+        e.tail = (u32)(((volatile SlotCtl*)p.sc)[vc->cur & p.kmask].word >> 32);
+        e.mode = vc->mode;
+        e.far_min = vc->far_min;
+        e.pad = 0;
+        p.trace[tn] = e;
+        vc->trace_n = tn + 1;
+      }
       __threadfence();
       atomicAdd(&c->bar_gen, 1u);
     } else {
       u32 ns = 32;
       while (ld_acquire_u32(&c->bar_gen) == gen) {
         __nanosleep(ns);
-        if (ns < 256) ns <<= 1;
+        if (ns < 128) ns <<= 1;
       }
     }
     __threadfence();
@@ -533,30 +646,39 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
 template <bool F32, bool PRO>
 __device__ void phase1(const Params& p, Smem& sm) {
   const u32 slot = sm.cur & p.kmask, lim = sm.lim;
+  SlotCtl* sc = p.sc + slot;
   u64* q = p.items + (u64)slot * p.cap;
   const u32 G = gridDim.x;
+  u32 my_next = 0, my_end = 0;  // thread 0: claimed ticket range
   for (;;) {
     if (threadIdx.x == 0) {
-      u32 n = 0, h = 0, ns = 32;
+      u32 n = 0, h = 0, ns = 32, waited = 0;
       for (;;) {
-        const u64 wv = ld_relaxed_u64(p.word + slot);
+        const u64 wv = ld_relaxed_u64(&sc->word);
         const u32 tail = min((u32)(wv >> 32), p.cap);
-        h = ld_relaxed_u32(p.head + slot);
-        if (h < tail) {
-          const u32 avail = tail - h;
-          u32 want = (avail + G - 1) / G;
-          want = max(want, 16u);
-          want = min(want, p.claim_max);
-          n = min(avail, want);
-          if (atomicCAS(p.head + slot, h, h + n) == h) break;
-          continue;
+        if (my_next >= my_end && my_end < p.cap) {
+          // claim size grows with the queue: small early (spread work), up to claim_max
+          u32 c = min(max(tail / (2 * G), 8u), p.claim_max);
+          my_next = atomicAdd(&sc->head, c);
+          my_end = my_next + c;
+        }
+        const u32 avail_end = min(my_end, tail);
+        const u32 avail = my_next < avail_end ? avail_end - my_next : 0u;
+        const u32 full = min(my_end - my_next, (u32)DS_THREADS);
+        // take a full batch at once; a partial one only after a short wait
+        if (avail && (avail >= full || avail >= 64u || waited > 2000u)) {
+          n = min(avail, (u32)DS_THREADS);
+          h = my_next;
+          my_next += n;
+          break;
         }
         if ((u32)wv == 0) {  // quiescent: nothing pending anywhere
           n = 0;
           break;
         }
         __nanosleep(ns);
-        if (ns < 512) ns <<= 1;
+        waited += ns;
+        if (ns < 256) ns <<= 1;
       }
       sm.claim_n = n;
       sm.claim_h = h;
@@ -566,9 +688,10 @@ __device__ void phase1(const Params& p, Smem& sm) {
     if (n == 0) break;
     const u32 h = sm.claim_h;
     u64 it = SENTINEL;
-    const bool has = threadIdx.x < n;
+    const u32 my = (threadIdx.x & 31) * DS_WARPS + (threadIdx.x >> 5);  // spread over warps
+    const bool has = my < n;
     if (has) {
-      u64* e = q + h + threadIdx.x;
+      u64* e = q + h + my;
       u32 ns = 16;
       while ((it = ld_relaxed_u64(e)) == SENTINEL) {  // reserved, not yet written
         __nanosleep(ns);
@@ -576,7 +699,7 @@ __device__ void phase1(const Params& p, Smem& sm) {
       }
     }
     process_batch<F32, PRO, 1>(p, sm, it, has, lim, SRC_QUEUE, slot);
-    if (threadIdx.x == 0) atomicAdd(p.word + slot, (u64)0 - (u64)n);  // completion
+    if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
   }
 }
 
@@ -587,8 +710,9 @@ __device__ void phase2(const Params& p, Smem& sm) {
   const u32 p2e = sm.p2_end;
   const u32 G = gridDim.x;
   const u32 span = sm.p2_end - sm.p2_begin;
-  const u32 CL = min(max((span + G - 1) / G, 16u), p.claim_max);
+  const u32 CL = min(max((span + 2 * G - 1) / (2 * G), 16u), p.claim_max);
   Ctl* c = p.ctl;
+  u32 hub_next = 0, hub_end = 0;  // thread 0: hub ticket
   for (;;) {
     if (threadIdx.x == 0) {
       u32 n = 0, h = 0, src = 0, ns = 32;
@@ -597,29 +721,29 @@ __device__ void phase2(const Params& p, Smem& sm) {
           h = atomicAdd(&c->p2_head, CL);
           if (h < p2e) {
             n = min(CL, p2e - h);
-            src = 1;
+            src = SRC_STATIC;
             break;
           }
         }
         const u64 wv = ld_relaxed_u64(&c->hub_word);
         const u32 tail = min((u32)(wv >> 32), p.hub_cap);
-        const u32 hh = ld_relaxed_u32(&c->hub_head);
-        if (hh < tail) {
-          const u32 nn = min(tail - hh, 2u);
-          if (atomicCAS(&c->hub_head, hh, hh + nn) == hh) {
-            h = hh;
-            n = nn;
-            src = 2;
-            break;
-          }
-          continue;
+        if (hub_next >= hub_end && hub_end < p.hub_cap && hub_end <= tail) {
+          hub_next = atomicAdd(&c->hub_head, 1u);  // one 4096-arc chunk per ticket
+          hub_end = hub_next + 1;
+        }
+        if (hub_next < hub_end && hub_next < tail) {
+          h = hub_next;
+          n = 1;
+          hub_next = hub_end;
+          src = SRC_HUB;
+          break;
         }
         if ((u32)wv == 0) {
           n = 0;
           break;
         }
         __nanosleep(ns);
-        if (ns < 512) ns <<= 1;
+        if (ns < 256) ns <<= 1;
       }
       sm.claim_n = n;
       sm.claim_h = h;
@@ -630,14 +754,15 @@ __device__ void phase2(const Params& p, Smem& sm) {
     if (n == 0) break;
     const u32 h = sm.claim_h, src = sm.claim_src;
     u64 it = SENTINEL;
-    const bool has = threadIdx.x < n;
+    const u32 my = (threadIdx.x & 31) * DS_WARPS + (threadIdx.x >> 5);  // spread over warps
+    const bool has = my < n;
     if (has) {
       if (src == SRC_STATIC) {
-        u64* e = q + h + threadIdx.x;
+        u64* e = q + h + my;
         it = ld_relaxed_u64(e);
         st_relaxed_u64(e, SENTINEL);  // recycle the queue entry
       } else {
-        u64* e = p.hub_items + h + threadIdx.x;
+        u64* e = p.hub_items + h + my;
         u32 ns = 16;
         while ((it = ld_relaxed_u64(e)) == SENTINEL) {
           __nanosleep(ns);
@@ -656,7 +781,7 @@ __device__ void rescan_clear(const Params& p) {
   const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
   const i64 nt = (i64)gridDim.x * blockDim.x;
   for (u32 s = 0; s < p.K; ++s) {
-    const u32 tail = min((u32)(ld_relaxed_u64(p.word + s) >> 32), p.cap);
+    const u32 tail = min((u32)(ld_relaxed_u64(&p.sc[s].word) >> 32), p.cap);
     u64* q = p.items + (u64)s * p.cap;
     for (i64 i = t; i < tail; i += nt) st_relaxed_u64(q + i, SENTINEL);
   }
@@ -668,16 +793,20 @@ __device__ void rescan_fill(const Params& p, Smem& sm) {
   const u32 base = sm.cur, lim = sm.lim;
   const i64 t0 = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL;
   const i64 nt = (i64)gridDim.x * blockDim.x;
+  const u32 inf = F32 ? 0x7F800000u : NONE;
   for (i64 b = t0; b < p.V; b += nt) {
     const i64 v = b + lane_id();
-    bool want = false;
-    u32 d = NONE;
+    bool want[UNROLL] = {};
+    u32 vv[UNROLL] = {}, dd[UNROLL] = {};
     if (v < p.V) {
-      d = ld_cg(p.dist + v);
-      want = d != (F32 ? 0x7F800000u : NONE) && bucket_of<F32>(p, d) >= base;
+      const u32 d = ld_cg(p.dist + v);
+      want[0] = d != inf && bucket_of<F32>(p, d) >= base;
+      vv[0] = (u32)v;
+      dd[0] = d;
     }
-    warp_push<F32>(p, sm, lim, want, (u32)v, d, NONE);
+    stage_pushes<F32>(p, sm, lim, NONE, want, vv, dd);
   }
+  if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
 }
 
 // Sweep fall-back for a bucket whose queue lost work (capacity): Bellman-Ford
@@ -712,13 +841,16 @@ __device__ void sweep(const Params& p, Smem& sm) {
 }
 
 template <bool F32, bool PRO>
-__global__ void __launch_bounds__(DS_THREADS, 2) k_delta_step(Params p) {
+__global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) {
   __shared__ Smem sm;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    TraceEnt e = {globaltimer(), 99u, 0u, 0u, 0u, 0u, 0u};
+    p.trace[0] = e;
+    p.ctl->trace_n = 1;
+  }
   if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
+  if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
-    sm.wl_n = 0;
-    sm.wl_next = 0;
-    sm.cl_n = 0;
     volatile Ctl* vc = p.ctl;
     sm.mode = vc->mode;
     sm.cur = vc->cur;
@@ -766,16 +898,16 @@ __global__ void k_fill_u32(u32* __restrict__ a, i64 n, u32 v) {
 __global__ void k_seed(Params p, u32 src) {
   const u32 t = threadIdx.x;
   for (u32 s = t; s < p.K; s += blockDim.x) {
-    p.word[s] = 0;
-    p.head[s] = 0;
-    p.p2[s] = 0;
+    p.sc[s].word = 0;
+    p.sc[s].head = 0;
+    p.sc[s].p2 = 0;
   }
   if (t < ST_N) p.stats[t] = 0;
   __syncthreads();
   if (t == 0) {
     p.dist[src] = 0;
     p.items[0] = (u64)src;  // (d=0 << 32) | src in bucket 0, slot 0
-    p.word[0] = (1ULL << 32) | 1ULL;
+    p.sc[0].word = (1ULL << 32) | 1ULL;
     Ctl* c = p.ctl;
     c->cur = 0;
     c->lim = p.K - 1;
@@ -792,6 +924,7 @@ __global__ void k_seed(Params p, u32 src) {
     c->sweeps = 0;
     c->hub_word = 0;
     c->hub_head = 0;
+    c->trace_n = 0;
   }
 }
 

@@ -51,12 +51,11 @@ struct sssp_graph_s {
   u32* dist = nullptr;
   u32* xd = nullptr;
   Ctl* ctl = nullptr;
-  u64* word = nullptr;
-  u32* head = nullptr;
-  u32* p2 = nullptr;
+  SlotCtl* sc = nullptr;
   u64* items = nullptr;
   u64* hub_items = nullptr;
   unsigned long long* stats = nullptr;
+  TraceEnt* trace = nullptr;
   u32 K_alloc = 0, cap_alloc = 0, hub_cap = 0;
   u32 K_used = 0;
   bool need_full_reset = true;
@@ -157,6 +156,7 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
     CG(cudaMalloc(&g->xd, sizeof(u32) * V));
     CG(cudaMalloc(&g->ctl, sizeof(Ctl)));
     CG(cudaMalloc(&g->stats, sizeof(unsigned long long) * ST_N));
+    CG(cudaMalloc(&g->trace, sizeof(TraceEnt) * TRACE_CAP));
     CG(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
     CG(cudaMemsetAsync(g->stats, 0, sizeof(unsigned long long) * ST_N, s));
     for (int i = 0; i < 4; ++i) CG(cudaEventCreate(&g->ev[i]));
@@ -212,8 +212,8 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   DeviceGuard dg(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
-  void* ptrs[] = {g->rowp, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->word,
-                  g->head, g->p2, g->items, g->hub_items, g->stats};
+  void* ptrs[] = {g->rowp, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
+                  g->items, g->hub_items, g->stats, g->trace};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& e : g->ev)
@@ -429,17 +429,12 @@ static sssp_status ensure_run_buffers(sssp_graph_t g, u32 K, u32 cap) {
   const u32 hub_cap = (u32)std::min<i64>(g->A / 2048 + 4096, 0x7FFFFFFF);
   if (K > g->K_alloc || cap != g->cap_alloc) {
     if (g->items) CU(cudaFree(g->items));
-    if (g->word) CU(cudaFree(g->word));
-    if (g->head) CU(cudaFree(g->head));
-    if (g->p2) CU(cudaFree(g->p2));
+    if (g->sc) CU(cudaFree(g->sc));
     g->items = nullptr;
-    g->word = nullptr;
-    g->head = nullptr;
-    g->p2 = nullptr;
+    g->sc = nullptr;
     CU(cudaMalloc(&g->items, sizeof(u64) * (size_t)K * cap));
-    CU(cudaMalloc(&g->word, sizeof(u64) * K));
-    CU(cudaMalloc(&g->head, sizeof(u32) * K));
-    CU(cudaMalloc(&g->p2, sizeof(u32) * K));
+    CU(cudaMalloc(&g->sc, sizeof(SlotCtl) * K));
+    CU(cudaMemsetAsync(g->sc, 0, sizeof(SlotCtl) * K, s));
     g->K_alloc = K;
     g->cap_alloc = cap;
     g->need_full_reset = true;
@@ -498,12 +493,11 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.dist = g->dist;
   p.xd = g->xd;
   p.ctl = g->ctl;
-  p.word = g->word;
-  p.head = g->head;
-  p.p2 = g->p2;
+  p.sc = g->sc;
   p.items = g->items;
   p.hub_items = g->hub_items;
   p.stats = g->stats;
+  p.trace = g->trace;
   p.V = (u32)g->V;
   p.K = K;
   p.kmask = K - 1;
@@ -717,6 +711,26 @@ extern "C" sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_
   if (reset) {
     g->kt_total_ms = 0.0;
     g->kt_launches = 0;
+  }
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
+                                      int64_t* n_entries) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!n_entries || (max_entries > 0 && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad trace buffer");
+  static_assert(sizeof(sssp_trace_entry) == sizeof(TraceEnt), "trace layout");
+  DeviceGuard dg(g->device);
+  Ctl c;
+  CU(cudaMemcpyAsync(&c, g->ctl, sizeof c, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaStreamSynchronize(g->stream));
+  const int64_t n = std::min<int64_t>(c.trace_n, TRACE_CAP);
+  *n_entries = n;
+  const int64_t k = std::min<int64_t>(n, std::max<int64_t>(max_entries, 0));
+  if (k > 0) {
+    CU(cudaMemcpyAsync(out, g->trace, sizeof(TraceEnt) * k, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
   }
   return SSSP_OK;
 }

@@ -1,0 +1,64 @@
+"""Run one SSSP on a config and print the device-side scheduler timeline.
+
+python tools/trace_run.py --config C4 [--delta 32] [--runs 3] [--param k=v]"""
+import argparse
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+NAMES = {0: "P1", 1: "P2", 2: "RC", 3: "RF", 4: "SL", 5: "SH", 99: "start"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--scale", type=int, default=None)
+    ap.add_argument("--delta", type=float, nargs="*", default=None)
+    ap.add_argument("--runs", type=int, default=3)
+    ap.add_argument("--no-reorder", action="store_true")
+    ap.add_argument("--param", action="append", default=[])
+    ap.add_argument("--quiet", action="store_true")
+    a = ap.parse_args()
+    import torch
+    import paper_conf_icppw_zhangczsdhay23_b200 as sssp
+
+    over = {"scale": a.scale} if a.scale else {}
+    t = time.time()
+    c = dict(gen.CONFIGS[a.config])
+    c.update(over)
+    g = gen.kronecker(c["scale"], c["edgefactor"], c["seed"], c["weights"]) if c["kind"] == "kron" else gen.make_config(a.config)
+    print(f"gen {time.time()-t:.1f}s V={g.V} A={g.A}", flush=True)
+    G = sssp.Graph(g.row, g.col, g.w)
+    for kv in a.param:
+        k, v = kv.split("=")
+        G.set_param(getattr(sssp, "SSSP_PARAM_" + k.upper()), int(v))
+    if not a.no_reorder:
+        G.reorder()
+        print("reorder_ms", G.stats()["reorder_ms"])
+    srcs = gen.sample_sources(g, 8, seed=7)
+    for delta in (a.delta or [c["delta"]]):
+        for r in range(a.runs):
+            G.run(int(srcs[r % len(srcs)]), delta)
+            torch.cuda.synchronize()
+            st = G.stats()
+            print(f"delta={delta} run {r}: {st['run_ms']:.3f} ms  GTEPS={g.m/st['run_ms']/1e6:.2f}  "
+                  f"upd={st['updates']} light={st['light_arcs']} heavy={st['heavy_arcs']} "
+                  f"settled={st['vertices_settled']} stale={st['stale_items']} chunks={st['hub_chunks']} "
+                  f"bins t/w/c={st['bin_thread']}/{st['bin_warp']}/{st['bin_cta']} buckets={st['buckets']} "
+                  f"rescans={st['rescans']} reach={st['reachable']}", flush=True)
+        if not a.quiet:
+            tr = G.trace()
+            prev = 0.0
+            for e in tr:
+                print(f"  {e['t_us']:10.1f} us (+{e['t_us']-prev:8.1f})  {NAMES.get(e['which'], e['which']):5s} "
+                      f"cur={e['cur']} tail={e['tail']} mode={e['mode']}")
+                prev = e["t_us"]
+
+
+if __name__ == "__main__":
+    main()
