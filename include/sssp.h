@@ -151,7 +151,9 @@ typedef enum {
     SSSP_PARAM_RING_SLOTS = 0,     /* K bucket queues, power of two in [4,64]; 0 = auto [0] */
     SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
     SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (1.25 V + 64Ki) [0] */
-    SSSP_PARAM_CLAIM_MAX = 3       /* max queue entries one CTA claims at once (1..256) [256] */
+    SSSP_PARAM_CLAIM_MAX = 3,      /* max queue entries one CTA claims at once (1..256) [256] */
+    SSSP_PARAM_L2_PERSIST = 4      /* 1: keep dist[] in a persisting L2 window (raises the
+                                      device's persisting-L2 limit; never lowers it) [1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 
@@ -175,6 +177,11 @@ typedef struct sssp_trace_entry {
 } sssp_trace_entry;
 sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
                            int64_t* n_entries);
+
+/* Diagnostics of the last run: summed SM cycles of thread 0 of every
+ * persistent CTA in [claim, stage, task, tail, grid-barrier] plus the number
+ * of batches and of 128-arc tasks (7 values). */
+sssp_status sssp_get_profile(sssp_graph_t g, uint64_t* out, int n);
 
 /* Library/device info: number of SMs of the handle's device. */
 int sssp_device_sm_count(sssp_graph_t g);

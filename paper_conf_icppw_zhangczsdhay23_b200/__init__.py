@@ -41,6 +41,7 @@ SSSP_PARAM_RING_SLOTS = 0
 SSSP_PARAM_CTAS_PER_SM = 1
 SSSP_PARAM_SLOT_CAPACITY = 2
 SSSP_PARAM_CLAIM_MAX = 3
+SSSP_PARAM_L2_PERSIST = 4
 
 INF_U32 = 0xFFFFFFFF
 
@@ -49,7 +50,7 @@ EXPORTS = (
     "sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
-    "sssp_kernel_time", "sssp_get_trace",
+    "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile",
 )
 
 
@@ -94,6 +95,8 @@ class sssp_trace_entry(ctypes.Structure):
 
 _lib.sssp_get_trace.argtypes = [_P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]
 _lib.sssp_get_trace.restype = _I
+_lib.sssp_get_profile.argtypes = [_P, _P, _I]
+_lib.sssp_get_profile.restype = _I
 for _n in ("sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
            "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param"):
     getattr(_lib, _n).restype = _I
@@ -231,6 +234,13 @@ def sssp_get_trace(h, max_entries=4096):
     return out
 
 
+def sssp_get_profile(h):
+    """Cycle accounting of the last run (thread 0 of every persistent CTA)."""
+    out = np.zeros(7, dtype=np.uint64)
+    _check(_lib.sssp_get_profile(h, out.ctypes.data, 7), "sssp_get_profile")
+    return dict(zip(("claim", "stage", "task", "tail", "barrier", "batches", "tasks"), out.tolist()))
+
+
 def sssp_device_sm_count(h):
     return int(_lib.sssp_device_sm_count(h))
 
@@ -293,6 +303,9 @@ class Graph:
 
     def kernel_time(self, reset=False):
         return sssp_kernel_time(self.h, reset)
+
+    def profile(self):
+        return sssp_get_profile(self.h)
 
     def trace(self):
         return sssp_get_trace(self.h)

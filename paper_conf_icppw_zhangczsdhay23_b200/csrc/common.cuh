@@ -46,6 +46,22 @@ __device__ __forceinline__ void st_relaxed_u32(u32* p, u32 v) {
   asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+// Bulk prefetch of a contiguous global range into L2 (sm_90+; no registers,
+// no completion tracking). Used to start the arc stream of every claimed
+// vertex while the batch is still being staged.
+__device__ __forceinline__ void prefetch_l2(const void* p, u32 bytes) {
+  const uintptr_t a = (uintptr_t)p & ~(uintptr_t)15;
+  const uintptr_t e = ((uintptr_t)p + bytes + 15) & ~(uintptr_t)15;
+  if (e > a)
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((u32)(e - a)) : "memory");
+}
+
+__device__ __forceinline__ u64 policy_evict_last() {
+  u64 pol;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+
 __device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31u; }
 __device__ __forceinline__ u32 lanemask_lt() {
   u32 m;

@@ -49,6 +49,9 @@ constexpr u32 HUB_CHUNK = 4096;
 #ifndef SSSP_PROBE_L1
 #define SSSP_PROBE_L1 1  // dist probes through L1 (a stale value is a safe filter)
 #endif
+#ifndef SSSP_PREFETCH
+#define SSSP_PREFETCH 1  // L2 bulk prefetch of each claimed vertex's arc range
+#endif
 constexpr int UNROLL = SSSP_UNROLL;
 constexpr u64 SENTINEL = ~0ULL;
 constexpr u32 NONE = 0xFFFFFFFFu;
@@ -78,6 +81,14 @@ enum {
   ST_BIN_T,
   ST_BIN_W,
   ST_BIN_C,
+  // cycle accounting of thread 0 of every CTA (diagnostics, sssp_get_profile)
+  ST_P_CLAIM,  // waiting for / claiming queue entries
+  ST_P_STAGE,  // batch decode + task-pool staging (until the pool barrier)
+  ST_P_TASK,   // warp 0 in the task loop
+  ST_P_TAIL,   // warp 0 after its last task until the batch barrier (flush + wait)
+  ST_P_BAR,    // grid barriers
+  ST_P_NB,     // batches
+  ST_P_NT,     // tasks
   ST_N
 };
 
@@ -153,6 +164,7 @@ struct Smem {
   u32 sb_off[DS_WARPS][32];
   u32 sb_d[DS_WARPS][32];
   u32 sb_total[DS_WARPS];
+  u32 sb_toff[DS_WARPS + 1];  // first thread-bin task of each warp
   u32 scan_ws[DS_WARPS];
   u32 rl_n, rl_tasks, task_next;
   u64 pb[DS_WARPS][PB_CAP];  // staged pushes (d << 32 | v), bucket resolved at flush
@@ -167,14 +179,53 @@ struct Smem {
 // Filter probe of dist[] before the atomicMin (Alg. 1 l.2). Any value ever
 // stored in dist[v] is >= its current value, so a stale (L1-cached) read can
 // only cause an extra atomic, never a missed improvement.
-__device__ __forceinline__ u32 ld_probe(const u32* p) {
-#if SSSP_PROBE_L1
+__device__ __forceinline__ u32 ld_probe(const u32* p, bool pred, u64 pol) {
   u32 v;
-  asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(v) : "l"(p));
-  return v;
+#if SSSP_PROBE_L1
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n mov.b32 %0, 0;\n"
+      " @q ld.global.ca.L2::cache_hint.u32 %0, [%1], %3;\n}"
+      : "=r"(v)
+      : "l"(p), "r"((u32)pred), "l"(pol));
 #else
-  return __ldcg(p);
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n mov.b32 %0, 0;\n"
+      " @q ld.global.cg.L2::cache_hint.u32 %0, [%1], %3;\n}"
+      : "=r"(v)
+      : "l"(p), "r"((u32)pred), "l"(pol));
 #endif
+  return v;
+}
+
+// Predicated arc load (streamed: L1 bypass, L2 evict-first). {0,0} if !pred.
+__device__ __forceinline__ uint2 ld_arc(const uint2* p, bool pred, u64 pol) {
+  uint2 v;
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n mov.b32 %0, 0;\n mov.b32 %1, 0;\n"
+      " @q ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %4;\n}"
+      : "=r"(v.x), "=r"(v.y)
+      : "l"(p), "r"((u32)pred), "l"(pol));
+  return v;
+}
+
+// Predicated atomicMin keeping dist[] L2-resident (evict_last). Returns the
+// old value, or 0 when !pred (so "nd < old" is false). All UNROLL atomics of
+// a group are issued before any result is consumed.
+__device__ __forceinline__ u32 atomic_min_keep(u32* p, u32 v, bool pred, u64 pol) {
+  u32 old;
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n mov.b32 %0, 0;\n"
+      " @q atom.relaxed.gpu.global.min.L2::cache_hint.u32 %0, [%1], %2, %4;\n}"
+      : "=r"(old)
+      : "l"(p), "r"(v), "r"((u32)pred), "l"(pol)
+      : "memory");
+  return old;
+}
+
+__device__ __forceinline__ u64 policy_evict_first() {
+  u64 pol;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
 }
 
 template <bool F32>
@@ -258,52 +309,78 @@ template <bool F32>
 __device__ __forceinline__ void stage_pushes(const Params& p, Smem& sm, u32 lim, u32 nearb,
                                              const bool (&want)[UNROLL], const u32 (&v)[UNROLL],
                                              const u32 (&nd)[UNROLL]) {
-  u32 c = 0;
+  u32 m[UNROLL], tot = 0;
 #pragma unroll
-  for (int k = 0; k < UNROLL; ++k) c += want[k];
-  if (!__any_sync(SSSP_FULL_MASK, c != 0)) return;
-  const u32 w = threadIdx.x >> 5;
-  u32 tot;
-  const u32 off = warp_exclusive_scan(c, &tot);
+  for (int k = 0; k < UNROLL; ++k) {
+    m[k] = __ballot_sync(SSSP_FULL_MASK, want[k]);
+    tot += __popc(m[k]);
+  }
+  if (!tot) return;
+  const u32 w = threadIdx.x >> 5, lt = lanemask_lt();
   if (sm.pb_n[w] + tot > PB_CAP) pb_flush<F32>(p, sm, lim, nearb);
-  u32 pos = sm.pb_n[w] + off;
+  u32 base = sm.pb_n[w];
 #pragma unroll
-  for (int k = 0; k < UNROLL; ++k)
-    if (want[k]) sm.pb[w][pos++] = ((u64)nd[k] << 32) | v[k];
+  for (int k = 0; k < UNROLL; ++k) {
+    if (want[k]) sm.pb[w][base + __popc(m[k] & lt)] = ((u64)nd[k] << 32) | v[k];
+    base += __popc(m[k]);
+  }
   __syncwarp();
-  if (lane_id() == 0) sm.pb_n[w] += tot;
+  if (lane_id() == 0) sm.pb_n[w] = base;
   __syncwarp();
 }
 
 // Relax UNROLL arcs per thread (independent loads in flight: arcs, then dist
 // probes, then atomics). PH 1 = light arcs, PH 2 = heavy arcs; without PRO the
 // light/heavy split is a per-arc predicate (the divergence PRO removes).
-template <bool F32, bool PRO, int PH>
-__device__ __forceinline__ void relax_group(const Params& p, Smem& sm, u32 lim, u32 nearb,
-                                            const u32 (&idx)[UNROLL], const bool (&valid)[UNROLL],
-                                            const u32 (&d)[UNROLL]) {
-  uint2 a[UNROLL];
-  u32 nd[UNROLL];
-  bool want[UNROLL];
+// Relax UNROLL arcs per thread in two steps so consecutive tasks overlap:
+// arcs_issue() starts the (streamed) arc loads of the next task before
+// relax_finish() of the current one waits on its dist probes and atomics.
+// PH 1 = light arcs, PH 2 = heavy arcs; without PRO the light/heavy split is
+// a per-arc predicate (the divergence PRO removes).
+__device__ __forceinline__ void arcs_issue(const Params& p, const u32 (&idx)[UNROLL],
+                                           const bool (&valid)[UNROLL], uint2 (&a)[UNROLL]) {
+  const u64 pol_stream = policy_evict_first();
 #pragma unroll
-  for (int k = 0; k < UNROLL; ++k) a[k] = valid[k] ? ld_stream_u2(p.arcs + idx[k]) : make_uint2(0, 0);
-  u32 cur[UNROLL];
+  for (int k = 0; k < UNROLL; ++k) a[k] = ld_arc(p.arcs + idx[k], valid[k], pol_stream);
+}
+
+template <bool F32, bool PRO, int PH>
+__device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim, u32 nearb,
+                                             const uint2 (&a)[UNROLL], const bool (&valid)[UNROLL],
+                                             const u32 (&d)[UNROLL]) {
+  const u64 pol_keep = policy_evict_last();
+  u32 nd[UNROLL], cur[UNROLL];
+  bool want[UNROLL];
+  bool of = false;
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     bool take = valid[k];
     if (!PRO) take = take && ((PH == 1) ? (a[k].y < p.delta_bits) : (a[k].y >= p.delta_bits));
+    if (F32) {
+      nd[k] = __float_as_uint(__fadd_rn(__uint_as_float(d[k]), __uint_as_float(a[k].y)));  // Alg. 1 l.1
+    } else {
+      const u64 sum = (u64)d[k] + a[k].y;  // exact; >= 0xFFFFFFFF is an overflow
+      const bool o = take && sum >= (u64)NONE;
+      of |= o;
+      take = take && !o;
+      nd[k] = (u32)sum;
+    }
     want[k] = take;
-    nd[k] = take ? relax_add<F32>(d[k], a[k].y, &p.ctl->err) : NONE;
-    cur[k] = take ? ld_probe(p.dist + a[k].x) : 0u;
+    cur[k] = ld_probe(p.dist + a[k].x, take, pol_keep);
   }
+  if (!F32 && of) atomicOr(&p.ctl->err, ERR_OVERFLOW);
+  u32 old[UNROLL];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     want[k] = want[k] && nd[k] < cur[k];  // check before the atomic (Alg. 1 l.2)
-    if (want[k]) want[k] = nd[k] < atomicMin(p.dist + a[k].x, nd[k]);  // Alg. 1 l.3
+    old[k] = atomic_min_keep(p.dist + a[k].x, nd[k], want[k], pol_keep);  // Alg. 1 l.3
   }
   u32 vv[UNROLL];
 #pragma unroll
-  for (int k = 0; k < UNROLL; ++k) vv[k] = a[k].x;
+  for (int k = 0; k < UNROLL; ++k) {
+    want[k] = want[k] && nd[k] < old[k];
+    vv[k] = a[k].x;
+  }
   stage_pushes<F32>(p, sm, lim, nearb, want, vv, nd);
 }
 
@@ -332,6 +409,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const bool sweep = src == SRC_SWEEP;
   const u32 nearb = sweep ? sm.cur : NONE;
+  const long long t_enter = tid == 0 ? clock64() : 0;
   bool small = false, listed = false;
   u32 beg = 0, len = 0, d = 0;
   u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0;
@@ -396,6 +474,9 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
       }
     }
   }
+#if SSSP_PREFETCH
+  if ((small || listed) && len) prefetch_l2(p.arcs + beg, len * (u32)sizeof(uint2));
+#endif
   // ---- stats (warp-aggregated)
   st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
   if (PH == 1) st_add(sm, ST_STALE, c_stale);
@@ -435,6 +516,11 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
       sm.rl_d[i] = d;
       sm.rl_toff[i] = off & 0xFFFFu;
     }
+    if (tid <= DS_WARPS) {  // thread-bin task offsets per warp
+      u32 a = 0;
+      for (int i = 0; i < (int)tid; ++i) a += (sm.sb_total[i] + TASK - 1) / TASK;
+      sm.sb_toff[tid] = a;
+    }
     if (tid == 0) {
       sm.rl_n = tot >> 16;
       sm.rl_tasks = tot & 0xFFFFu;
@@ -443,27 +529,30 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
     }
   }
   __syncthreads();  // task pool complete
+  long long t_pool = 0;
+  if (tid == 0) {
+    t_pool = clock64();
+    sm.st[ST_P_STAGE] += (unsigned long long)(t_pool - t_enter);
+    sm.st[ST_P_NB] += 1;
+  }
 
-  // small-task offsets per warp
-  u32 soff_w[DS_WARPS + 1];
-  soff_w[0] = 0;
-#pragma unroll
-  for (int i = 0; i < DS_WARPS; ++i) soff_w[i + 1] = soff_w[i] + (sm.sb_total[i] + TASK - 1) / TASK;
-  const u32 S = soff_w[DS_WARPS];
+  const u32 S = sm.sb_toff[DS_WARPS];
   const u32 ntask = S + sm.rl_tasks, nl = sm.rl_n;
-  for (;;) {
-    u32 t = 0;
-    if (lane == 0) t = atomicAdd(&sm.task_next, 1u);
-    t = __shfl_sync(SSSP_FULL_MASK, t, 0);
-    if (t >= ntask) break;
-    u32 idx[UNROLL];
-    bool valid[UNROLL];
-    u32 dd[UNROLL];
-    if (t < S) {  // thread-bin slice of warp ww
+  if (tid == 0) sm.st[ST_P_NT] += ntask;
+  // Task descriptor -> per-lane arc indices / distances (smem lookups only).
+  auto setup = [&](u32 t, u32 (&idx)[UNROLL], bool (&valid)[UNROLL], u32 (&dd)[UNROLL]) {
+    if (t >= ntask) {
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        valid[k] = false;
+        idx[k] = 0;
+        dd[k] = 0;
+      }
+    } else if (t < S) {  // thread-bin slice of warp ww
       u32 ww = 0;
 #pragma unroll
-      for (int i = 1; i < DS_WARPS; ++i) ww += (t >= soff_w[i]);
-      const u32 j0 = (t - soff_w[ww]) * TASK, total = sm.sb_total[ww];
+      for (int i = 1; i < DS_WARPS; ++i) ww += (t >= sm.sb_toff[i]);
+      const u32 j0 = (t - sm.sb_toff[ww]) * TASK, total = sm.sb_total[ww];
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
         const u32 j = j0 + k * 32 + lane;
@@ -497,10 +586,42 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
         dd[k] = dv;
       }
     }
-    relax_group<F32, PRO, PH>(p, sm, lim, nearb, idx, valid, dd);
+  };
+  auto claim = [&]() {
+    u32 t = 0;
+    if (lane == 0) t = atomicAdd(&sm.task_next, 1u);
+    return __shfl_sync(SSSP_FULL_MASK, t, 0);
+  };
+  u32 idx[UNROLL], dd[UNROLL];
+  bool valid[UNROLL];
+  uint2 a[UNROLL];
+  u32 t = claim();
+  setup(t, idx, valid, dd);
+  arcs_issue(p, idx, valid, a);
+  while (t < ntask) {
+    const u32 t2 = claim();
+    u32 idx2[UNROLL], dd2[UNROLL];
+    bool valid2[UNROLL];
+    uint2 a2[UNROLL];
+    setup(t2, idx2, valid2, dd2);
+    arcs_issue(p, idx2, valid2, a2);  // next task's arcs in flight ...
+    relax_finish<F32, PRO, PH>(p, sm, lim, nearb, a, valid, dd);  // ... while this one completes
+    t = t2;
+#pragma unroll
+    for (int k = 0; k < UNROLL; ++k) {
+      a[k] = a2[k];
+      valid[k] = valid2[k];
+      dd[k] = dd2[k];
+    }
+  }
+  long long t_task = 0;
+  if (tid == 0) {
+    t_task = clock64();
+    sm.st[ST_P_TASK] += (unsigned long long)(t_task - t_pool);
   }
   if (sm.pb_n[w]) pb_flush<F32>(p, sm, lim, nearb);  // publish before reporting completion
   __syncthreads();
+  if (tid == 0) sm.st[ST_P_TAIL] += (unsigned long long)(clock64() - t_task);
 }
 
 // --------------------------------------------------------- grid barrier ---
@@ -598,6 +719,7 @@ __device__ void decide(const Params& p, u32 which) {
 __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
   __syncthreads();
   if (threadIdx.x == 0) {
+    const long long t_b = clock64();
     Ctl* c = p.ctl;
     const u32 gen = ld_acquire_u32(&c->bar_gen);
     __threadfence();
@@ -638,6 +760,7 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
     sm.p2_begin = vc->p2_begin;
     sm.p2_end = vc->p2_end;
     sm.sweep_first = vc->sweep_first;
+    sm.st[ST_P_BAR] += (unsigned long long)(clock64() - t_b);
   }
   __syncthreads();
 }
@@ -652,6 +775,7 @@ __device__ void phase1(const Params& p, Smem& sm) {
   u32 my_next = 0, my_end = 0;  // thread 0: claimed ticket range
   for (;;) {
     if (threadIdx.x == 0) {
+      const long long t_c = clock64();
       u32 n = 0, h = 0, ns = 32, waited = 0;
       for (;;) {
         const u64 wv = ld_relaxed_u64(&sc->word);
@@ -682,6 +806,7 @@ __device__ void phase1(const Params& p, Smem& sm) {
       }
       sm.claim_n = n;
       sm.claim_h = h;
+      sm.st[ST_P_CLAIM] += (unsigned long long)(clock64() - t_c);
     }
     __syncthreads();
     const u32 n = sm.claim_n;
@@ -715,6 +840,7 @@ __device__ void phase2(const Params& p, Smem& sm) {
   u32 hub_next = 0, hub_end = 0;  // thread 0: hub ticket
   for (;;) {
     if (threadIdx.x == 0) {
+      const long long t_c = clock64();
       u32 n = 0, h = 0, src = 0, ns = 32;
       for (;;) {
         if (ld_relaxed_u32(&c->p2_head) < p2e) {
@@ -748,6 +874,7 @@ __device__ void phase2(const Params& p, Smem& sm) {
       sm.claim_n = n;
       sm.claim_h = h;
       sm.claim_src = src;
+      sm.st[ST_P_CLAIM] += (unsigned long long)(clock64() - t_c);
     }
     __syncthreads();
     const u32 n = sm.claim_n;

@@ -70,7 +70,9 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = 256;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = 256, p_l2 = 1;
+  i64 l2_window_bytes = -1;  // -1: not configured yet
+  float l2_hit_ratio = 1.f;
 };
 
 #define CU(call)                                                                       \
@@ -266,6 +268,11 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_SLOT_CAPACITY:
       if (v < 0 || v > 0x7FFFFFFFLL || (v != 0 && v < 4096)) return fail(SSSP_ERR_INVALID_ARGUMENT, "slot capacity 0 or in [4096, 2^31)");
       g->p_cap = v;
+      return SSSP_OK;
+    case SSSP_PARAM_L2_PERSIST:
+      if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "l2 persist is 0 or 1");
+      g->p_l2 = v;
+      g->l2_window_bytes = -1;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > DS_THREADS) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,256]");
@@ -481,6 +488,25 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   sssp_status st = ensure_run_buffers(g, K, cap);
   if (st) return st;
   g->K_used = K;
+  if (g->l2_window_bytes < 0) {
+    // Persisting L2 set-aside for dist[] (4 B per vertex). The set-aside is a
+    // device-wide limit; it is only ever raised, never lowered.
+    g->l2_window_bytes = 0;
+    int max_persist = 0, max_window = 0;
+    cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, g->device);
+    cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, g->device);
+    const i64 want = (i64)sizeof(u32) * g->V;
+    if (g->p_l2 && max_persist > 0 && max_window > 0) {
+      size_t cur = 0;
+      cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+      const size_t set_aside = (size_t)std::min<i64>(want, max_persist);
+      if (cur < set_aside) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, set_aside);
+      cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+      g->l2_window_bytes = std::min<i64>(want, max_window);
+      g->l2_hit_ratio = (float)std::min(1.0, (double)cur / (double)g->l2_window_bytes);
+    }
+    cudaGetLastError();
+  }
   ds_kernel_t kern = pick_kernel(f32, pro);
   int per_sm = 0;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, DS_THREADS, 0));
@@ -525,8 +551,31 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   g->ev_pending.emplace_back(e0, e1);
   CU(cudaEventRecord(e0, s));
   if (timed) CU(cudaEventRecord(g->ev[0], s));
-  void* args[] = {&p};
-  CU(cudaLaunchCooperativeKernel((const void*)kern, dim3(g->grid_ctas), dim3(DS_THREADS), args, 0, s));
+  // Cooperative launch (all CTAs co-resident: the grid barrier and the work
+  // queues need forward progress) with an L2 access-policy window that keeps
+  // dist[] persisting in L2 while arcs and queue entries stream through.
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(g->grid_ctas);
+  cfg.blockDim = dim3(DS_THREADS);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute attrs[2];
+  int na = 0;
+  attrs[na].id = cudaLaunchAttributeCooperative;
+  attrs[na].val.cooperative = 1;
+  ++na;
+  if (g->l2_window_bytes > 0) {
+    attrs[na].id = cudaLaunchAttributeAccessPolicyWindow;
+    attrs[na].val.accessPolicyWindow.base_ptr = g->dist;
+    attrs[na].val.accessPolicyWindow.num_bytes = (size_t)g->l2_window_bytes;
+    attrs[na].val.accessPolicyWindow.hitRatio = g->l2_hit_ratio;
+    attrs[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    attrs[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    ++na;
+  }
+  cfg.attrs = attrs;
+  cfg.numAttrs = na;
+  CU(cudaLaunchKernelEx(&cfg, kern, p));
   if (timed) CU(cudaEventRecord(g->ev[1], s));
   CU(cudaEventRecord(e1, s));
   g->run_timed = timed;
@@ -732,5 +781,17 @@ extern "C" sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int
     CU(cudaMemcpyAsync(out, g->trace, sizeof(TraceEnt) * k, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
   }
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_get_profile(sssp_graph_t g, uint64_t* out, int n) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out || n < 0) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad profile buffer");
+  DeviceGuard dg(g->device);
+  unsigned long long h[ST_N];
+  CU(cudaMemcpyAsync(h, g->stats, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaStreamSynchronize(g->stream));
+  for (int i = 0; i < n && i < (int)(ST_N - ST_P_CLAIM); ++i) out[i] = h[ST_P_CLAIM + i];
   return SSSP_OK;
 }

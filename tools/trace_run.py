@@ -51,6 +51,10 @@ def main():
                   f"settled={st['vertices_settled']} stale={st['stale_items']} chunks={st['hub_chunks']} "
                   f"bins t/w/c={st['bin_thread']}/{st['bin_warp']}/{st['bin_cta']} buckets={st['buckets']} "
                   f"rescans={st['rescans']} reach={st['reachable']}", flush=True)
+            pr = G.profile()
+            cyc = sum(pr[k] for k in ("claim", "stage", "task", "tail", "barrier"))
+            print("    profile %: " + " ".join(f"{k}={100*pr[k]/max(cyc,1):.1f}" for k in ("claim", "stage", "task", "tail", "barrier"))
+                  + f" batches={pr['batches']} tasks={pr['tasks']} avg_task_cyc(w0)={pr['task']/max(pr['tasks'],1)*1.0:.0f}", flush=True)
         if not a.quiet:
             tr = G.trace()
             prev = 0.0
