@@ -53,6 +53,16 @@ constexpr u32 HUB_CHUNK = 4096;
 #define SSSP_PREFETCH 1  // L2 bulk prefetch of each claimed vertex's arc range
 #endif
 constexpr int UNROLL = SSSP_UNROLL;
+#ifndef SSSP_IPT
+#define SSSP_IPT 2  // queue items decoded per thread per batch
+#endif
+constexpr int IPT = SSSP_IPT;
+#ifndef SSSP_CLAIM_MINPART
+#define SSSP_CLAIM_MINPART 64u  // take a partial batch once this many entries are ready ...
+#endif
+#ifndef SSSP_CLAIM_WAIT_NS
+#define SSSP_CLAIM_WAIT_NS 2000u  // ... or after waiting this long for a full one
+#endif
 constexpr u64 SENTINEL = ~0ULL;
 constexpr u32 NONE = 0xFFFFFFFFu;
 constexpr u32 CHUNK_FLAG = 0x80000000u;
@@ -147,6 +157,8 @@ struct Params {
 };
 
 constexpr u32 TASK = 32 * UNROLL;  // arcs per warp task
+constexpr u32 BATCH = DS_THREADS * IPT;  // queue items per CTA batch
+constexpr u32 SB_CAP = 32 * IPT;         // thread-bin entries per warp
 constexpr u32 PB_CAP = 256;        // staged pushes per warp (>= 32 * UNROLL)
 
 struct Smem {
@@ -156,16 +168,17 @@ struct Smem {
   // vertices and hub chunks: a 256..4096-arc vertex is spread over the CTA's
   // 8 warps = "CTA per vertex"; a 32..255-arc one takes 1-2 tasks = "warp per
   // vertex"). Any warp may run any task, so warps stay balanced.
-  u32 rl_beg[DS_THREADS];
-  u32 rl_len[DS_THREADS];
-  u32 rl_d[DS_THREADS];
-  u32 rl_toff[DS_THREADS + 1];
-  u32 sb_beg[DS_WARPS][32];
-  u32 sb_off[DS_WARPS][32];
-  u32 sb_d[DS_WARPS][32];
+  u32 rl_beg[BATCH];
+  u32 rl_len[BATCH];
+  u32 rl_d[BATCH];
+  u32 rl_toff[BATCH + 1];
+  u32 sb_beg[DS_WARPS][SB_CAP];
+  u32 sb_off[DS_WARPS][SB_CAP];
+  u32 sb_d[DS_WARPS][SB_CAP];
+  u32 sb_n[DS_WARPS];
   u32 sb_total[DS_WARPS];
   u32 sb_toff[DS_WARPS + 1];  // first thread-bin task of each warp
-  u32 scan_ws[DS_WARPS];
+  u64 scan_ws[DS_WARPS];
   u32 rl_n, rl_tasks, task_next;
   u64 pb[DS_WARPS][PB_CAP];  // staged pushes (d << 32 | v), bucket resolved at flush
   u32 pb_n[DS_WARPS];
@@ -399,22 +412,40 @@ __device__ __forceinline__ void item_range(const Params& p, u32 v, i64& b, i64& 
 }
 
 // ------------------------------------------------------------ batch -------
-// Process the CTA's claimed items (at most one per thread; has = holds one).
+// Batch item q (0 <= q < n) lives in thread (x % 8) * 32 + x / 8 of round
+// r = q / 256 (x = q % 256): consecutive items are spread over the 8 warps.
+__device__ __forceinline__ u32 batch_item_index(u32 r) {
+  return r * DS_THREADS + (threadIdx.x & 31) * DS_WARPS + (threadIdx.x >> 5);
+}
+
+// Process the CTA's claimed items (IPT per thread; has[i] = holds item i).
 // src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
 // phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
 // into the current bucket, hubs stay in the range list).
 template <bool F32, bool PRO, int PH>
-__device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it, bool has, u32 lim,
-                                              u32 src, u32 slot) {
+__device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u64 (&it)[IPT],
+                                              const bool (&has)[IPT], u32 lim, u32 src, u32 slot) {
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const bool sweep = src == SRC_SWEEP;
   const u32 nearb = sweep ? sm.cur : NONE;
   const long long t_enter = tid == 0 ? clock64() : 0;
-  bool small = false, listed = false;
-  u32 beg = 0, len = 0, d = 0;
-  u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0;
-  if (has) {
-    const u32 lo = (u32)it, hi = (u32)(it >> 32);
+  // ---- decode: all dist probes and row loads of the thread's items in flight at once
+  u32 cls[IPT], beg[IPT], len[IPT], d[IPT];
+  u32 cd[IPT];
+#pragma unroll
+  for (int i = 0; i < IPT; ++i) {
+    const u32 lo = (u32)it[i];
+    cls[i] = 0;
+    cd[i] = has[i] ? ld_cg(p.dist + (lo & ~CHUNK_FLAG)) : 0u;
+  }
+  u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0, c_t = 0;
+#pragma unroll
+  for (int i = 0; i < IPT; ++i) {
+    beg[i] = 0;
+    len[i] = 0;
+    d[i] = 0;
+    if (!has[i]) continue;
+    const u32 lo = (u32)it[i], hi = (u32)(it[i] >> 32);
     const bool is_chunk = (lo & CHUNK_FLAG) != 0;
     const u32 v = lo & ~CHUNK_FLAG;
     if (is_chunk) {
@@ -423,28 +454,25 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
         i64 rb, re;
         item_range<PRO, PH>(p, v, rb, re);
         const i64 b = rb + (i64)hi * HUB_CHUNK;
-        beg = (u32)b;
-        len = (u32)min((i64)HUB_CHUNK, re - b);
-        d = ld_cg(p.dist + v);  // current distance: a valid path length (<= spawning d)
-        c_arcs = len;
-        listed = true;
+        beg[i] = (u32)b;
+        len[i] = (u32)min((i64)HUB_CHUNK, re - b);
+        d[i] = cd[i];  // current distance: a valid path length (<= spawning d)
+        c_arcs += len[i];
+        cls[i] = 2;
       }
     } else {
-      const u32 cd = ld_cg(p.dist + v);
-      d = hi;
-      const bool live = (PH == 1) ? (d <= cd) : (d == cd);  // stale / settled-final filter
+      d[i] = hi;
+      const bool live = (PH == 1) ? (hi <= cd[i]) : (hi == cd[i]);  // stale / settled-final filter
       if (!live) {
-        c_stale = (PH == 1);
+        c_stale += (PH == 1);
       } else {
-        c_settled = 1;
+        c_settled += 1;
         i64 rb, re;
         item_range<PRO, PH>(p, v, rb, re);
         const i64 l = re - rb;
-        c_arcs = (u32)l;
         if (l > (i64)HUB_CHUNK && !sweep) {  // hub: ceil(l/4096) chunks any CTA may claim
           const u32 nc = (u32)((l + HUB_CHUNK - 1) / HUB_CHUNK);
-          c_chunks = nc;
-          c_arcs = 0;  // counted when the chunks run
+          c_chunks += nc;
           u64* word = (PH == 1) ? &p.sc[slot].word : &p.ctl->hub_word;
           u64* q = (PH == 1) ? p.items + (u64)slot * p.cap : p.hub_items;
           const u32 qcap = (PH == 1) ? p.cap : p.hub_cap;
@@ -461,60 +489,88 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
             }
           }
         } else if (l >= (i64)BIN_WARP) {
-          beg = (u32)rb;
-          len = (u32)l;
-          listed = true;
-          c_c = l >= (i64)BIN_CTA;
-          c_w = !c_c;
+          beg[i] = (u32)rb;
+          len[i] = (u32)l;
+          cls[i] = 2;
+          c_arcs += (u32)l;
+          if (l >= (i64)BIN_CTA)
+            ++c_c;
+          else
+            ++c_w;
         } else if (l > 0) {
-          small = true;
-          beg = (u32)rb;
-          len = (u32)l;
+          beg[i] = (u32)rb;
+          len[i] = (u32)l;
+          cls[i] = 1;
+          c_arcs += (u32)l;
+          ++c_t;
         }
       }
     }
   }
 #if SSSP_PREFETCH
-  if ((small || listed) && len) prefetch_l2(p.arcs + beg, len * (u32)sizeof(uint2));
+#pragma unroll
+  for (int i = 0; i < IPT; ++i)
+    if (cls[i]) prefetch_l2(p.arcs + beg[i], len[i] * (u32)sizeof(uint2));
 #endif
   // ---- stats (warp-aggregated)
   st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
   if (PH == 1) st_add(sm, ST_STALE, c_stale);
   st_add(sm, PH == 1 ? ST_LIGHT : ST_HEAVY, c_arcs);
   st_add(sm, ST_CHUNKS, c_chunks);
-  st_add(sm, ST_BIN_T, small ? 1u : 0u);
+  st_add(sm, ST_BIN_T, c_t);
   st_add(sm, ST_BIN_W, c_w);
   st_add(sm, ST_BIN_C, c_c);
 
-  // ---- stage: thread bin (warp prefix sum) and range list (block scan)
+  // ---- stage: thread bin (warp prefix sums) and range list (block scan)
   {
-    u32 stot;
-    const u32 soff = warp_exclusive_scan(small ? len : 0u, &stot);
-    sm.sb_beg[w][lane] = beg;
-    sm.sb_off[w][lane] = soff;  // monotone; zero-length lanes never own an arc
-    sm.sb_d[w][lane] = d;
-    const u32 x = listed ? ((1u << 16) | ((len + TASK - 1) / TASK)) : 0u;
-    u32 wt;
-    const u32 ex = warp_exclusive_scan(x, &wt);
+    u32 ns = 0, ls = 0, nl = 0, tl = 0;
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      ns += cls[i] == 1;
+      ls += cls[i] == 1 ? len[i] : 0u;
+      nl += cls[i] == 2;
+      tl += cls[i] == 2 ? (len[i] + TASK - 1) / TASK : 0u;
+    }
+    u32 tot_ns, tot_ls;
+    u32 pos = warp_exclusive_scan(ns, &tot_ns);
+    u32 off = warp_exclusive_scan(ls, &tot_ls);
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      if (cls[i] == 1) {
+        sm.sb_beg[w][pos] = beg[i];
+        sm.sb_off[w][pos] = off;
+        sm.sb_d[w][pos] = d[i];
+        ++pos;
+        off += len[i];
+      }
+    }
+    const u64 x = ((u64)nl << 32) | tl;
+    u64 wt;
+    const u64 ex = warp_exclusive_scan(x, &wt);
     if (lane == 31) {
       sm.scan_ws[w] = wt;
-      sm.sb_total[w] = stot;
+      sm.sb_n[w] = tot_ns;
+      sm.sb_total[w] = tot_ls;
     }
     __syncthreads();
-    u32 acc = 0, tot = 0;
+    u64 acc = 0, tot = 0;
 #pragma unroll
     for (int i = 0; i < DS_WARPS; ++i) {
-      const u32 s = sm.scan_ws[i];
-      if (i < (int)w) acc += s;
-      tot += s;
+      const u64 sv = sm.scan_ws[i];
+      if (i < (int)w) acc += sv;
+      tot += sv;
     }
-    const u32 off = ex + acc;
-    if (listed) {
-      const u32 i = off >> 16;
-      sm.rl_beg[i] = beg;
-      sm.rl_len[i] = len;
-      sm.rl_d[i] = d;
-      sm.rl_toff[i] = off & 0xFFFFu;
+    u32 li = (u32)((ex + acc) >> 32), lt = (u32)(ex + acc);
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      if (cls[i] == 2) {
+        sm.rl_beg[li] = beg[i];
+        sm.rl_len[li] = len[i];
+        sm.rl_d[li] = d[i];
+        sm.rl_toff[li] = lt;
+        ++li;
+        lt += (len[i] + TASK - 1) / TASK;
+      }
     }
     if (tid <= DS_WARPS) {  // thread-bin task offsets per warp
       u32 a = 0;
@@ -522,9 +578,9 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
       sm.sb_toff[tid] = a;
     }
     if (tid == 0) {
-      sm.rl_n = tot >> 16;
-      sm.rl_tasks = tot & 0xFFFFu;
-      sm.rl_toff[tot >> 16] = tot & 0xFFFFu;
+      sm.rl_n = (u32)(tot >> 32);
+      sm.rl_tasks = (u32)tot;
+      sm.rl_toff[(u32)(tot >> 32)] = (u32)tot;
       sm.task_next = 0;
     }
   }
@@ -552,15 +608,15 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, u64 it,
       u32 ww = 0;
 #pragma unroll
       for (int i = 1; i < DS_WARPS; ++i) ww += (t >= sm.sb_toff[i]);
-      const u32 j0 = (t - sm.sb_toff[ww]) * TASK, total = sm.sb_total[ww];
+      const u32 j0 = (t - sm.sb_toff[ww]) * TASK, total = sm.sb_total[ww], ne = sm.sb_n[ww];
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
         const u32 j = j0 + k * 32 + lane;
         valid[k] = j < total;
-        u32 o = 0;  // owner: last lane with sb_off <= j
+        u32 o = 0;  // owner: last entry with sb_off <= j
 #pragma unroll
-        for (u32 step = 16; step; step >>= 1)
-          if (sm.sb_off[ww][o + step] <= j) o += step;
+        for (u32 step = SB_CAP / 2; step; step >>= 1)
+          if (o + step < ne && sm.sb_off[ww][o + step] <= j) o += step;
         idx[k] = sm.sb_beg[ww][o] + (j - sm.sb_off[ww][o]);
         dd[k] = sm.sb_d[ww][o];
       }
@@ -788,10 +844,10 @@ __device__ void phase1(const Params& p, Smem& sm) {
         }
         const u32 avail_end = min(my_end, tail);
         const u32 avail = my_next < avail_end ? avail_end - my_next : 0u;
-        const u32 full = min(my_end - my_next, (u32)DS_THREADS);
+        const u32 full = min(my_end - my_next, BATCH);
         // take a full batch at once; a partial one only after a short wait
-        if (avail && (avail >= full || avail >= 64u || waited > 2000u)) {
-          n = min(avail, (u32)DS_THREADS);
+        if (avail && (avail >= full || avail >= SSSP_CLAIM_MINPART || waited > SSSP_CLAIM_WAIT_NS)) {
+          n = min(avail, BATCH);
           h = my_next;
           my_next += n;
           break;
@@ -812,15 +868,21 @@ __device__ void phase1(const Params& p, Smem& sm) {
     const u32 n = sm.claim_n;
     if (n == 0) break;
     const u32 h = sm.claim_h;
-    u64 it = SENTINEL;
-    const u32 my = (threadIdx.x & 31) * DS_WARPS + (threadIdx.x >> 5);  // spread over warps
-    const bool has = my < n;
-    if (has) {
-      u64* e = q + h + my;
+    u64 it[IPT];
+    bool has[IPT];
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      const u32 my = batch_item_index(i);
+      has[i] = my < n;
+      it[i] = has[i] ? ld_relaxed_u64(q + h + my) : SENTINEL;
+    }
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
       u32 ns = 16;
-      while ((it = ld_relaxed_u64(e)) == SENTINEL) {  // reserved, not yet written
+      while (has[i] && it[i] == SENTINEL) {  // reserved, not yet written
         __nanosleep(ns);
         if (ns < 256) ns <<= 1;
+        it[i] = ld_relaxed_u64(q + h + batch_item_index(i));
       }
     }
     process_batch<F32, PRO, 1>(p, sm, it, has, lim, SRC_QUEUE, slot);
@@ -835,7 +897,7 @@ __device__ void phase2(const Params& p, Smem& sm) {
   const u32 p2e = sm.p2_end;
   const u32 G = gridDim.x;
   const u32 span = sm.p2_end - sm.p2_begin;
-  const u32 CL = min(max((span + 2 * G - 1) / (2 * G), 16u), p.claim_max);
+  const u32 CL = min(max((span + 2 * G - 1) / (2 * G), 16u), min(p.claim_max, BATCH));
   Ctl* c = p.ctl;
   u32 hub_next = 0, hub_end = 0;  // thread 0: hub ticket
   for (;;) {
@@ -880,23 +942,25 @@ __device__ void phase2(const Params& p, Smem& sm) {
     const u32 n = sm.claim_n;
     if (n == 0) break;
     const u32 h = sm.claim_h, src = sm.claim_src;
-    u64 it = SENTINEL;
-    const u32 my = (threadIdx.x & 31) * DS_WARPS + (threadIdx.x >> 5);  // spread over warps
-    const bool has = my < n;
-    if (has) {
-      if (src == SRC_STATIC) {
-        u64* e = q + h + my;
-        it = ld_relaxed_u64(e);
-        st_relaxed_u64(e, SENTINEL);  // recycle the queue entry
-      } else {
-        u64* e = p.hub_items + h + my;
-        u32 ns = 16;
-        while ((it = ld_relaxed_u64(e)) == SENTINEL) {
-          __nanosleep(ns);
-          if (ns < 256) ns <<= 1;
-        }
-        st_relaxed_u64(e, SENTINEL);
+    u64 it[IPT];
+    bool has[IPT];
+    u64* const base_q = src == SRC_STATIC ? q + h : p.hub_items + h;
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      const u32 my = batch_item_index(i);
+      has[i] = my < n;
+      it[i] = has[i] ? ld_relaxed_u64(base_q + my) : SENTINEL;
+    }
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      if (!has[i]) continue;
+      u32 ns = 16;
+      while (it[i] == SENTINEL) {  // hub chunks may be reserved but not yet written
+        __nanosleep(ns);
+        if (ns < 256) ns <<= 1;
+        it[i] = ld_relaxed_u64(base_q + batch_item_index(i));
       }
+      st_relaxed_u64(base_q + batch_item_index(i), SENTINEL);  // recycle the queue entry
     }
     process_batch<F32, PRO, 2>(p, sm, it, has, lim, src, slot);
     if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
@@ -945,22 +1009,27 @@ __device__ void sweep(const Params& p, Smem& sm) {
   const u32 cur = sm.cur, lim = sm.lim;
   const bool first = sm.sweep_first != 0;
   const u32 inf = F32 ? 0x7F800000u : NONE;
-  for (i64 base = (i64)blockIdx.x * DS_THREADS; base < p.V; base += (i64)gridDim.x * DS_THREADS) {
-    const i64 v = base + threadIdx.x;
-    bool has = false;
-    u64 it = SENTINEL;
-    if (v < p.V) {
-      const u32 d = ld_cg(p.dist + v);
-      if (d != inf && bucket_of<F32>(p, d) == cur) {
-        if (PH == 1) {
-          if (first || d < ld_cg(p.xd + v)) {
-            st_relaxed_u32(p.xd + v, d);
-            has = true;
+  for (i64 base = (i64)blockIdx.x * BATCH; base < p.V; base += (i64)gridDim.x * BATCH) {
+    bool has[IPT];
+    u64 it[IPT];
+#pragma unroll
+    for (int i = 0; i < IPT; ++i) {
+      const i64 v = base + batch_item_index(i);
+      has[i] = false;
+      it[i] = SENTINEL;
+      if (v < p.V) {
+        const u32 d = ld_cg(p.dist + v);
+        if (d != inf && bucket_of<F32>(p, d) == cur) {
+          if (PH == 1) {
+            if (first || d < ld_cg(p.xd + v)) {
+              st_relaxed_u32(p.xd + v, d);
+              has[i] = true;
+            }
+          } else {
+            has[i] = true;
           }
-        } else {
-          has = true;
+          it[i] = ((u64)d << 32) | (u64)v;
         }
-        it = ((u64)d << 32) | (u64)v;
       }
     }
     process_batch<F32, PRO, PH>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);

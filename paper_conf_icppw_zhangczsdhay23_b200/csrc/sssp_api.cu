@@ -70,7 +70,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = 256, p_l2 = 1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -275,7 +275,7 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       g->l2_window_bytes = -1;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
-      if (v < 1 || v > DS_THREADS) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,256]");
+      if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
       g->p_claim = v;
       return SSSP_OK;
   }
