@@ -54,9 +54,14 @@ constexpr u32 HUB_CHUNK = 4096;
 #endif
 constexpr int UNROLL = SSSP_UNROLL;
 #ifndef SSSP_IPT
-#define SSSP_IPT 2  // queue items decoded per thread per batch
+#define SSSP_IPT 2  // queue items decoded per thread per phase-1 batch
+#endif
+#ifndef SSSP_IPT2
+#define SSSP_IPT2 2  // ... per phase-2 batch (static, all items ready)
 #endif
 constexpr int IPT = SSSP_IPT;
+constexpr int IPT2 = SSSP_IPT2;
+constexpr int IPT_MAX = IPT > IPT2 ? IPT : IPT2;
 #ifndef SSSP_CLAIM_MINPART
 #define SSSP_CLAIM_MINPART 64u  // take a partial batch once this many entries are ready ...
 #endif
@@ -157,9 +162,13 @@ struct Params {
 };
 
 constexpr u32 TASK = 32 * UNROLL;  // arcs per warp task
-constexpr u32 BATCH = DS_THREADS * IPT;  // queue items per CTA batch
-constexpr u32 SB_CAP = 32 * IPT;         // thread-bin entries per warp
-constexpr u32 PB_CAP = 256;        // staged pushes per warp (>= 32 * UNROLL)
+constexpr u32 BATCH = DS_THREADS * IPT;        // queue items per phase-1 CTA batch
+constexpr u32 BATCH_MAX = DS_THREADS * IPT_MAX;
+constexpr u32 SB_CAP = 32 * IPT_MAX;           // thread-bin entries per warp
+#ifndef SSSP_PB_CAP
+#define SSSP_PB_CAP 256u
+#endif
+constexpr u32 PB_CAP = SSSP_PB_CAP;  // staged pushes per warp (>= 32 * UNROLL)
 
 struct Smem {
   // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
@@ -168,10 +177,10 @@ struct Smem {
   // vertices and hub chunks: a 256..4096-arc vertex is spread over the CTA's
   // 8 warps = "CTA per vertex"; a 32..255-arc one takes 1-2 tasks = "warp per
   // vertex"). Any warp may run any task, so warps stay balanced.
-  u32 rl_beg[BATCH];
-  u32 rl_len[BATCH];
-  u32 rl_d[BATCH];
-  u32 rl_toff[BATCH + 1];
+  u32 rl_beg[BATCH_MAX];
+  u32 rl_len[BATCH_MAX];
+  u32 rl_d[BATCH_MAX];
+  u32 rl_toff[BATCH_MAX + 1];
   u32 sb_beg[DS_WARPS][SB_CAP];
   u32 sb_off[DS_WARPS][SB_CAP];
   u32 sb_d[DS_WARPS][SB_CAP];
@@ -422,25 +431,25 @@ __device__ __forceinline__ u32 batch_item_index(u32 r) {
 // src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
 // phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
 // into the current bucket, hubs stay in the range list).
-template <bool F32, bool PRO, int PH>
-__device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u64 (&it)[IPT],
-                                              const bool (&has)[IPT], u32 lim, u32 src, u32 slot) {
+template <bool F32, bool PRO, int PH, int N>
+__device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u64 (&it)[N],
+                                              const bool (&has)[N], u32 lim, u32 src, u32 slot) {
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const bool sweep = src == SRC_SWEEP;
   const u32 nearb = sweep ? sm.cur : NONE;
   const long long t_enter = tid == 0 ? clock64() : 0;
   // ---- decode: all dist probes and row loads of the thread's items in flight at once
-  u32 cls[IPT], beg[IPT], len[IPT], d[IPT];
-  u32 cd[IPT];
+  u32 cls[N], beg[N], len[N], d[N];
+  u32 cd[N];
 #pragma unroll
-  for (int i = 0; i < IPT; ++i) {
+  for (int i = 0; i < N; ++i) {
     const u32 lo = (u32)it[i];
     cls[i] = 0;
     cd[i] = has[i] ? ld_cg(p.dist + (lo & ~CHUNK_FLAG)) : 0u;
   }
   u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0, c_t = 0;
 #pragma unroll
-  for (int i = 0; i < IPT; ++i) {
+  for (int i = 0; i < N; ++i) {
     beg[i] = 0;
     len[i] = 0;
     d[i] = 0;
@@ -509,7 +518,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   }
 #if SSSP_PREFETCH
 #pragma unroll
-  for (int i = 0; i < IPT; ++i)
+  for (int i = 0; i < N; ++i)
     if (cls[i]) prefetch_l2(p.arcs + beg[i], len[i] * (u32)sizeof(uint2));
 #endif
   // ---- stats (warp-aggregated)
@@ -525,7 +534,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   {
     u32 ns = 0, ls = 0, nl = 0, tl = 0;
 #pragma unroll
-    for (int i = 0; i < IPT; ++i) {
+    for (int i = 0; i < N; ++i) {
       ns += cls[i] == 1;
       ls += cls[i] == 1 ? len[i] : 0u;
       nl += cls[i] == 2;
@@ -535,7 +544,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
     u32 pos = warp_exclusive_scan(ns, &tot_ns);
     u32 off = warp_exclusive_scan(ls, &tot_ls);
 #pragma unroll
-    for (int i = 0; i < IPT; ++i) {
+    for (int i = 0; i < N; ++i) {
       if (cls[i] == 1) {
         sm.sb_beg[w][pos] = beg[i];
         sm.sb_off[w][pos] = off;
@@ -562,7 +571,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
     }
     u32 li = (u32)((ex + acc) >> 32), lt = (u32)(ex + acc);
 #pragma unroll
-    for (int i = 0; i < IPT; ++i) {
+    for (int i = 0; i < N; ++i) {
       if (cls[i] == 2) {
         sm.rl_beg[li] = beg[i];
         sm.rl_len[li] = len[i];
@@ -885,7 +894,7 @@ __device__ void phase1(const Params& p, Smem& sm) {
         it[i] = ld_relaxed_u64(q + h + batch_item_index(i));
       }
     }
-    process_batch<F32, PRO, 1>(p, sm, it, has, lim, SRC_QUEUE, slot);
+    process_batch<F32, PRO, 1, IPT>(p, sm, it, has, lim, SRC_QUEUE, slot);
     if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
   }
 }
@@ -897,7 +906,7 @@ __device__ void phase2(const Params& p, Smem& sm) {
   const u32 p2e = sm.p2_end;
   const u32 G = gridDim.x;
   const u32 span = sm.p2_end - sm.p2_begin;
-  const u32 CL = min(max((span + 2 * G - 1) / (2 * G), 16u), min(p.claim_max, BATCH));
+  const u32 CL = min(max((span + 2 * G - 1) / (2 * G), 16u), (u32)(DS_THREADS * IPT2));
   Ctl* c = p.ctl;
   u32 hub_next = 0, hub_end = 0;  // thread 0: hub ticket
   for (;;) {
@@ -942,17 +951,17 @@ __device__ void phase2(const Params& p, Smem& sm) {
     const u32 n = sm.claim_n;
     if (n == 0) break;
     const u32 h = sm.claim_h, src = sm.claim_src;
-    u64 it[IPT];
-    bool has[IPT];
+    u64 it[IPT2];
+    bool has[IPT2];
     u64* const base_q = src == SRC_STATIC ? q + h : p.hub_items + h;
 #pragma unroll
-    for (int i = 0; i < IPT; ++i) {
+    for (int i = 0; i < IPT2; ++i) {
       const u32 my = batch_item_index(i);
       has[i] = my < n;
       it[i] = has[i] ? ld_relaxed_u64(base_q + my) : SENTINEL;
     }
 #pragma unroll
-    for (int i = 0; i < IPT; ++i) {
+    for (int i = 0; i < IPT2; ++i) {
       if (!has[i]) continue;
       u32 ns = 16;
       while (it[i] == SENTINEL) {  // hub chunks may be reserved but not yet written
@@ -962,7 +971,7 @@ __device__ void phase2(const Params& p, Smem& sm) {
       }
       st_relaxed_u64(base_q + batch_item_index(i), SENTINEL);  // recycle the queue entry
     }
-    process_batch<F32, PRO, 2>(p, sm, it, has, lim, src, slot);
+    process_batch<F32, PRO, 2, IPT2>(p, sm, it, has, lim, src, slot);
     if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
   }
 }
@@ -1032,7 +1041,7 @@ __device__ void sweep(const Params& p, Smem& sm) {
         }
       }
     }
-    process_batch<F32, PRO, PH>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);
+    process_batch<F32, PRO, PH, IPT>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);
   }
 }
 
