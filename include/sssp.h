@@ -179,8 +179,10 @@ sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_en
                            int64_t* n_entries);
 
 /* Diagnostics of the last run: summed SM cycles of thread 0 of every
- * persistent CTA in [claim, stage, task, tail, grid-barrier] plus the number
- * of batches and of 128-arc tasks (7 values). */
+ * persistent CTA in [claim, stage, task, tail, grid-barrier], the number of
+ * batches and of warp tasks, then (diagnostics builds with SSSP_LAT=1 only,
+ * else 0) warp-0 cycles waiting for arcs, dist probes, atomics, staging and
+ * the number of tasks measured (12 values). */
 sssp_status sssp_get_profile(sssp_graph_t g, uint64_t* out, int n);
 
 /* Library/device info: number of SMs of the handle's device. */

@@ -236,9 +236,11 @@ def sssp_get_trace(h, max_entries=4096):
 
 def sssp_get_profile(h):
     """Cycle accounting of the last run (thread 0 of every persistent CTA)."""
-    out = np.zeros(7, dtype=np.uint64)
-    _check(_lib.sssp_get_profile(h, out.ctypes.data, 7), "sssp_get_profile")
-    return dict(zip(("claim", "stage", "task", "tail", "barrier", "batches", "tasks"), out.tolist()))
+    names = ("claim", "stage", "task", "tail", "barrier", "batches", "tasks",
+             "lat_arc", "lat_probe", "lat_atom", "lat_stage", "lat_n", "atoms")
+    out = np.zeros(len(names), dtype=np.uint64)
+    _check(_lib.sssp_get_profile(h, out.ctypes.data, len(names)), "sssp_get_profile")
+    return dict(zip(names, out.tolist()))
 
 
 def sssp_device_sm_count(h):

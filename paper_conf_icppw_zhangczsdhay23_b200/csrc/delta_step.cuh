@@ -52,6 +52,9 @@ constexpr u32 HUB_CHUNK = 4096;
 #ifndef SSSP_PREFETCH
 #define SSSP_PREFETCH 1  // L2 bulk prefetch of each claimed vertex's arc range
 #endif
+#ifndef SSSP_LAT
+#define SSSP_LAT 0  // per-stage latency accounting in the task loop (diagnostics build)
+#endif
 constexpr int UNROLL = SSSP_UNROLL;
 #ifndef SSSP_IPT
 #define SSSP_IPT 2  // queue items decoded per thread per phase-1 batch
@@ -104,6 +107,12 @@ enum {
   ST_P_BAR,    // grid barriers
   ST_P_NB,     // batches
   ST_P_NT,     // tasks
+  ST_L_ARC,    // warp 0: cycles waiting for a task's arcs (issued one task ahead)
+  ST_L_PROBE,  // ... for its dist probes
+  ST_L_ATOM,   // ... for its atomics
+  ST_L_STAGE,  // ... staging the pushes
+  ST_L_N,      // tasks measured
+  ST_ATOMS,    // atomicMin issued (diagnostics builds)
   ST_N
 };
 
@@ -374,6 +383,14 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
   u32 nd[UNROLL], cur[UNROLL];
   bool want[UNROLL];
   bool of = false;
+#if SSSP_LAT
+  long long t0 = 0, t1 = 0, t2 = 0, t3 = 0;
+  if (threadIdx.x == 0) {
+    t0 = clock64();
+    asm volatile("" ::"r"(a[0].x), "r"(a[UNROLL - 1].x));
+    t1 = clock64();
+  }
+#endif
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     bool take = valid[k];
@@ -391,19 +408,48 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
     cur[k] = ld_probe(p.dist + a[k].x, take, pol_keep);
   }
   if (!F32 && of) atomicOr(&p.ctl->err, ERR_OVERFLOW);
+#if SSSP_LAT
+  if (threadIdx.x == 0) {
+    asm volatile("" ::"r"(cur[0]), "r"(cur[UNROLL - 1]));
+    t2 = clock64();
+  }
+  u32 n_atoms = 0;
+#endif
   u32 old[UNROLL];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     want[k] = want[k] && nd[k] < cur[k];  // check before the atomic (Alg. 1 l.2)
+#if SSSP_LAT
+    n_atoms += want[k];
+#endif
     old[k] = atomic_min_keep(p.dist + a[k].x, nd[k], want[k], pol_keep);  // Alg. 1 l.3
   }
+#if SSSP_LAT
+  st_add(sm, ST_ATOMS, n_atoms);
+#endif
   u32 vv[UNROLL];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     want[k] = want[k] && nd[k] < old[k];
     vv[k] = a[k].x;
   }
+#if SSSP_LAT
+  if (threadIdx.x == 0) {
+    asm volatile("" ::"r"(old[0]), "r"(old[UNROLL - 1]));
+    t3 = clock64();
+  }
+#endif
   stage_pushes<F32>(p, sm, lim, nearb, want, vv, nd);
+#if SSSP_LAT
+  if (threadIdx.x == 0) {
+    const long long t4 = clock64();
+    sm.st[ST_L_ARC] += (unsigned long long)(t1 - t0);
+    sm.st[ST_L_PROBE] += (unsigned long long)(t2 - t1);
+    sm.st[ST_L_ATOM] += (unsigned long long)(t3 - t2);
+    sm.st[ST_L_STAGE] += (unsigned long long)(t4 - t3);
+    sm.st[ST_L_N] += 1;
+  }
+#endif
 }
 
 // Range of an item for phase PH: PRO -> light [start, heavy) / heavy [heavy, end);

@@ -55,6 +55,10 @@ def main():
             cyc = sum(pr[k] for k in ("claim", "stage", "task", "tail", "barrier"))
             print("    profile %: " + " ".join(f"{k}={100*pr[k]/max(cyc,1):.1f}" for k in ("claim", "stage", "task", "tail", "barrier"))
                   + f" batches={pr['batches']} tasks={pr['tasks']} avg_task_cyc(w0)={pr['task']/max(pr['tasks'],1)*1.0:.0f}", flush=True)
+            if pr["lat_n"]:
+                n = pr["lat_n"]
+                print(f"    task latency (cycles, warp 0): arc={pr['lat_arc']/n:.0f} probe={pr['lat_probe']/n:.0f} "
+                      f"atom={pr['lat_atom']/n:.0f} stage={pr['lat_stage']/n:.0f} atomics_issued={pr['atoms']}", flush=True)
         if not a.quiet:
             tr = G.trace()
             prev = 0.0
