@@ -183,4 +183,94 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(Fields<NF> in, Fields
   }
 }
 
+// Stable scatter through shared memory: the tile is first reordered by digit
+// in shared memory (same stable ranks as k_rs_scatter), then written out in
+// digit runs so consecutive threads store consecutive global addresses.
+// Dynamic shared memory: NF * RS_TILE * 4 bytes of staging.
+template <int NF>
+__global__ void __launch_bounds__(RS_THREADS) k_rs_scatter_smem(Fields<NF> in, Fields<NF> out, int kf,
+                                                                i64 n, int sh,
+                                                                const u32* __restrict__ hist_scan,
+                                                                u32 ntiles) {
+  extern __shared__ u32 stage[];  // [NF][RS_TILE]
+  __shared__ u32 wcnt[RS_THREADS / 32][256];
+  __shared__ u32 gbase[256];
+  __shared__ u32 dstart[257];
+  const u32 w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+#pragma unroll
+  for (int i = 0; i < RS_THREADS / 32; ++i) wcnt[i][threadIdx.x] = 0;
+  gbase[threadIdx.x] = hist_scan[(i64)threadIdx.x * ntiles + blockIdx.x];
+  __syncthreads();
+  const i64 tbase = (i64)blockIdx.x * RS_TILE;
+  const i64 base = tbase + (i64)w * RS_WARP_ELEMS;
+  u32 dig[RS_ROUNDS];
+  u32 rnk[RS_ROUNDS];
+#pragma unroll
+  for (int r = 0; r < RS_ROUNDS; ++r) {
+    const i64 i = base + r * 32 + lane;
+    const bool valid = i < n;
+    const u32 d = valid ? (in.f[kf][i] >> sh) & 255u : 0u;
+    dig[r] = valid ? d : 256u;
+    const u32 m = __ballot_sync(SSSP_FULL_MASK, valid);
+    u32 b = 0, peers = 0;
+    if (valid) {
+      peers = __match_any_sync(m, d);
+      b = wcnt[w][d];
+    }
+    __syncwarp();
+    if (valid && lane == (u32)(__ffs(peers) - 1)) wcnt[w][d] = b + __popc(peers);
+    __syncwarp();
+    rnk[r] = b + __popc(peers & lanemask_lt());
+  }
+  __syncthreads();
+  {  // per digit: exclusive scan over warps, tile total
+    u32 run = 0;
+#pragma unroll
+    for (int i = 0; i < RS_THREADS / 32; ++i) {
+      u32 c = wcnt[i][threadIdx.x];
+      wcnt[i][threadIdx.x] = run;
+      run += c;
+    }
+    dstart[threadIdx.x] = run;  // tile count of this digit (scanned below)
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {  // exclusive scan of 256 digit counts by one warp
+    u32 v[8], t = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      v[j] = dstart[threadIdx.x * 8 + j];
+      t += v[j];
+    }
+    u32 tot;
+    u32 ex = warp_exclusive_scan(t, &tot);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const u32 c = v[j];
+      dstart[threadIdx.x * 8 + j] = ex;
+      ex += c;
+    }
+    if (threadIdx.x == 31) dstart[256] = tot;
+  }
+  __syncthreads();
+  // scatter into shared memory in digit order
+#pragma unroll
+  for (int r = 0; r < RS_ROUNDS; ++r) {
+    if (dig[r] < 256u) {
+      const i64 i = base + r * 32 + lane;
+      const u32 lp = dstart[dig[r]] + wcnt[w][dig[r]] + rnk[r];
+#pragma unroll
+      for (int k = 0; k < NF; ++k) stage[k * RS_TILE + lp] = in.f[k][i];
+    }
+  }
+  __syncthreads();
+  // coalesced write-out of the digit runs
+  const u32 cnt = dstart[256];
+  for (u32 lp = threadIdx.x; lp < cnt; lp += RS_THREADS) {
+    const u32 d = (stage[kf * RS_TILE + lp] >> sh) & 255u;
+    const u32 gp = gbase[d] + (lp - dstart[d]);
+#pragma unroll
+    for (int k = 0; k < NF; ++k) out.f[k][gp] = stage[k * RS_TILE + lp];
+  }
+}
+
 }  // namespace sssp

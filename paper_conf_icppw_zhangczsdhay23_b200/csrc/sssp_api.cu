@@ -290,7 +290,13 @@ static sssp_status radix_pass(sssp_graph_t g, Fields<NF>& a, Fields<NF>& b, int 
   const u32 ntiles = (u32)((n + RS_TILE - 1) / RS_TILE);
   k_rs_hist<<<ntiles, RS_THREADS, 0, s>>>(a.f[kf], n, sh, hist, ntiles);
   scan_exclusive_rec<u32>(hist, hist, (i64)256 * ntiles, tmp, s);
-  k_rs_scatter<NF><<<ntiles, RS_THREADS, 0, s>>>(a, b, kf, n, sh, hist, ntiles);
+  const size_t smem = (size_t)NF * RS_TILE * sizeof(u32);
+  static bool attr_set = false;  // per NF instantiation
+  if (!attr_set) {
+    CU(cudaFuncSetAttribute(k_rs_scatter_smem<NF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr_set = true;
+  }
+  k_rs_scatter_smem<NF><<<ntiles, RS_THREADS, smem, s>>>(a, b, kf, n, sh, hist, ntiles);
   std::swap(a, b);
   CU(cudaGetLastError());
   return SSSP_OK;
@@ -356,8 +362,25 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   if (A > 0) {
     // a2+a3: one stable LSD radix sort of all arcs by (new src, w, new dst)
     for (int i = 0; i < 6; ++i) CU(cudaMallocAsync(&f[i], sizeof(u32) * A, s));
-    k_expand_arcs<<<grid_for((i64)V * 32), 256, 0, s>>>(g->rowp, g->arcs, V, deg ? g->old2new : nullptr,
-                                                       f[0], f[1], f[2]);
+    // arcs of vertices with <= EXPAND_HUB arcs: warp-flattened; hubs: 4096-arc
+    // chunks over all blocks. The hub count is bounded by A / EXPAND_HUB, so
+    // the chunk scan runs over that capacity with no host round trip.
+    const u32 nh_cap = (u32)(A / EXPAND_HUB + 1);
+    u32 *hubs = nullptr, *cst = nullptr, *ctmp = nullptr;
+    CU(cudaMallocAsync(&hubs, sizeof(u32) * (nh_cap + 1), s));
+    CU(cudaMallocAsync(&cst, sizeof(u32) * (nh_cap + 1), s));
+    CU(cudaMallocAsync(&ctmp, sizeof(u32) * scan_tmp_elems(nh_cap + 1), s));
+    CU(cudaMemsetAsync(hubs + nh_cap, 0, sizeof(u32), s));
+    k_list_hubs<<<grid_for(V), 256, 0, s>>>(g->rowp, V, hubs, hubs + nh_cap);
+    k_expand_arcs_flat<<<grid_for(V), 256, 0, s>>>(g->rowp, g->arcs, V, deg ? g->old2new : nullptr,
+                                                   f[0], f[1], f[2]);
+    k_hub_chunks<<<(nh_cap + 256) / 256, 256, 0, s>>>(g->rowp, hubs, hubs + nh_cap, nh_cap, cst);
+    scan_exclusive_rec<u32>(cst, cst, (i64)nh_cap + 1, ctmp, s);
+    k_expand_hubs<<<g->num_sms * 8, 256, 0, s>>>(g->rowp, g->arcs, hubs, nh_cap, cst,
+                                                 deg ? g->old2new : nullptr, f[0], f[1], f[2]);
+    CU(cudaFreeAsync(hubs, s));
+    CU(cudaFreeAsync(cst, s));
+    CU(cudaFreeAsync(ctmp, s));
     CU(cudaGetLastError());
     Fields<3> a{{f[0], f[1], f[2]}}, b{{f[3], f[4], f[5]}};
     const int vb = bits_for((u64)(V - 1));
