@@ -39,6 +39,8 @@ struct sssp_graph_s {
   i64 V = 0, A = 0;
   sssp_weight_type wtype = SSSP_WEIGHT_U32;
   longlong2* rowp = nullptr;  // [V+1] {start, heavy}
+  uint2* rowc = nullptr;      // [V+1] compact copy for the persistent kernel
+  bool rowc_valid = false;
   uint2* arcs = nullptr;      // [A]
   u32 maxw_bits = 0;
   u32* old2new = nullptr;  // null until PRO_DEGREE
@@ -153,6 +155,7 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
       }                                                                                 \
     }
     CG(cudaMalloc(&g->rowp, sizeof(longlong2) * (V + 1)));
+    CG(cudaMalloc(&g->rowc, sizeof(uint2) * (V + 1)));
     CG(cudaMalloc(&g->arcs, sizeof(uint2) * std::max<i64>(A, 1)));
     CG(cudaMalloc(&g->dist, sizeof(u32) * V));
     CG(cudaMalloc(&g->xd, sizeof(u32) * V));
@@ -214,7 +217,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   DeviceGuard dg(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
-  void* ptrs[] = {g->rowp, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
+  void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
                   g->items, g->hub_items, g->stats, g->trace};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -415,6 +418,7 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   }
   g->pro_flags |= flags;
   g->heavy_valid = false;
+  g->rowc_valid = false;
   g->have_result = false;
   g->reorder_timed = true;
   return SSSP_OK;
@@ -498,6 +502,12 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
     CU(cudaGetLastError());
     g->heavy_valid = true;
     g->heavy_bits = dp.delta_bits;
+    g->rowc_valid = false;
+  }
+  if (!g->rowc_valid) {
+    k_make_rowc<<<grid_for(g->V + 1), 256, 0, s>>>(g->rowp, g->V, g->rowc);
+    CU(cudaGetLastError());
+    g->rowc_valid = true;
   }
   // ring size: enough slots for the farthest heavy push (+ the recycled slot)
   u32 K = (u32)g->p_ring;
@@ -537,7 +547,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   if (g->p_ctas > 0) per_sm = std::min<int>(per_sm, (int)g->p_ctas);
   g->grid_ctas = per_sm * g->num_sms;
   Params p;
-  p.rowp = g->rowp;
+  p.rowc = g->rowc;
   p.arcs = g->arcs;
   p.dist = g->dist;
   p.xd = g->xd;
