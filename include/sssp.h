@@ -150,7 +150,7 @@ sssp_status sssp_export_csr(sssp_graph_t g, double delta, int64_t* rowlist, uint
 typedef enum {
     SSSP_PARAM_RING_SLOTS = 0,     /* K bucket queues, power of two in [4,64]; 0 = auto [0] */
     SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
-    SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (1.25 V + 64Ki) [0] */
+    SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (2.5 V + 64Ki) [0] */
     SSSP_PARAM_CLAIM_MAX = 3,      /* max queue entries one CTA claims at once (1..1024) [1024] */
     SSSP_PARAM_L2_PERSIST = 4      /* 1: keep dist[] in a persisting L2 window (raises the
                                       device's persisting-L2 limit; never lowers it) [1] */

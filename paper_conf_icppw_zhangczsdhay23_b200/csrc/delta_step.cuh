@@ -200,8 +200,6 @@ struct Smem {
   u32 rl_n, rl_tasks, task_next;
   u64 pb[DS_WARPS][PB_CAP];  // staged pushes (d << 32 | v), bucket resolved at flush
   u32 pb_n[DS_WARPS];
-  u32 fl_cnt[DS_WARPS][32];  // pb_flush: entries per bucket offset
-  u32 fl_pos[DS_WARPS][32];  // pb_flush: next reserved queue index per bucket offset
   unsigned long long st[ST_N];
   u32 claim_h, claim_n, claim_src;
   // control snapshot
@@ -295,57 +293,42 @@ __device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
 // ring horizon or a full queue are dropped and recorded in far_min. In the
 // sweep fall-back (nearb != NONE) entries of bucket nearb mark xd[] instead.
 template <bool F32>
-__device__ __noinline__ void pb_flush(const Params& p, Smem& sm, u32 lim, u32 nearb) {
+__device__ __noinline__ void pb_flush(const Params p, Smem& sm, u32 lim, u32 nearb) {
   const u32 lane = lane_id(), w = threadIdx.x >> 5;
   const u32 n = sm.pb_n[w];
-  const u32 cur = sm.cur;
   if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)n);
-  // pass 1: count entries per bucket offset (rel < 32), handle the rest
-  sm.fl_cnt[w][lane] = 0;
-  __syncwarp();
-  for (u32 i = lane; i < n; i += 32) {
-    const u64 e = sm.pb[w][i];
+  for (u32 i0 = 0; i0 < n; i0 += 32) {
+    const u32 i = i0 + lane;
+    bool ok = i < n;
+    const u64 e = ok ? sm.pb[w][i] : 0ULL;
     const u32 v = (u32)e, nd = (u32)(e >> 32);
-    const u32 x = bucket_of<F32>(p, nd);
-    if (x == nearb) {
+    const u32 x = ok ? bucket_of<F32>(p, nd) : 0u;
+    if (ok && x == nearb) {
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
-    } else if (x > lim) {  // beyond the ring horizon: rescan later
+      ok = false;
+    }
+    if (ok && x > lim) {  // beyond the ring horizon: rescan later
       atomicMin(&p.ctl->far_min, x);
-    } else if (x - cur < 32u) {
-      atomicAdd(&sm.fl_cnt[w][x - cur], 1u);
-    } else {  // rare: more than 31 buckets ahead: reserve one slot directly
-      const u32 sl = x & p.kmask;
-      const u32 idx = (u32)(atomicAdd(&p.sc[sl].word, (1ULL << 32) | 1ULL) >> 32);
+      ok = false;
+    }
+    const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
+    if (ok) {
+      const u32 s = x & p.kmask;
+      const u32 peers = __match_any_sync(m, s);
+      const u32 leader = __ffs(peers) - 1;
+      const u32 cnt = __popc(peers);
+      u64 old = 0;
+      if (lane == leader) old = atomicAdd(&p.sc[s].word, ((u64)cnt << 32) | cnt);
+      old = __shfl_sync(peers, old, leader);
+      const u32 idx = (u32)(old >> 32) + __popc(peers & lanemask_lt());
       if (idx < p.cap) {
-        st_relaxed_u64(p.items + (u64)sl * p.cap + idx, e);
-      } else {
-        atomicAdd(&p.sc[sl].word, ~0ULL);
+        st_relaxed_u64(p.items + (u64)s * p.cap + idx, e);
+      } else {  // queue full: undo the pending count, recover later
+        atomicAdd(&p.sc[s].word, ~0ULL);
         atomicMin(&p.ctl->far_min, x);
       }
     }
-  }
-  __syncwarp();
-  // one global reservation per bucket, all issued together (one round trip)
-  {
-    const u32 c = sm.fl_cnt[w][lane];
-    u32 base = 0;
-    if (c) base = (u32)(atomicAdd(&p.sc[(cur + lane) & p.kmask].word, ((u64)c << 32) | c) >> 32);
-    sm.fl_pos[w][lane] = base;
-    if (c && base + c > p.cap) {  // queue full: undo the lost pending counts, recover later
-      const u32 lost = base >= p.cap ? c : base + c - p.cap;
-      atomicAdd(&p.sc[(cur + lane) & p.kmask].word, (u64)0 - (u64)lost);
-      atomicMin(&p.ctl->far_min, cur + lane);
-    }
-  }
-  __syncwarp();
-  // pass 2: write entries into their reserved ranges
-  for (u32 i = lane; i < n; i += 32) {
-    const u64 e = sm.pb[w][i];
-    const u32 x = bucket_of<F32>(p, (u32)(e >> 32));
-    if (x == nearb || x > lim || x - cur >= 32u) continue;
-    const u32 idx = atomicAdd(&sm.fl_pos[w][x - cur], 1u);
-    if (idx < p.cap) st_relaxed_u64(p.items + (u64)(x & p.kmask) * p.cap + idx, e);
   }
   __syncwarp();
   if (lane == 0) sm.pb_n[w] = 0;

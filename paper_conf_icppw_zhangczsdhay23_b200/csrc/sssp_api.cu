@@ -517,7 +517,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
     while (K < need && K < 32) K <<= 1;
   }
   u32 cap = (u32)g->p_cap;
-  if (cap == 0) cap = (u32)std::min<i64>(g->V + g->V / 4 + 65536, 0x7FFFFFFF);
+  if (cap == 0) cap = (u32)std::min<i64>(2 * g->V + g->V / 2 + 65536, 0x7FFFFFFF);  // 2.5 V: far buckets collect repeated improvements
   sssp_status st = ensure_run_buffers(g, K, cap);
   if (st) return st;
   g->K_used = K;
