@@ -130,6 +130,7 @@ typedef struct sssp_stats {
     uint64_t buckets;          /* phase-1 epochs run (buckets + reopenings) */
     uint64_t rescans;          /* overflow fall-back rescans of dist[] */
     uint64_t reachable;        /* vertices with a finite distance (filled by sssp_distances) */
+    uint64_t levels;           /* extra phase-1 frontier levels (SSSP_PARAM_SYNC=1 only) */
     uint32_t ring_slots;       /* K: bucket-queue ring size used */
     uint32_t grid_ctas;        /* persistent grid size */
     float run_ms;              /* device time of the last sssp_run (CUDA events) */
@@ -152,8 +153,13 @@ typedef enum {
     SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
     SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (2.5 V + 64Ki) [0] */
     SSSP_PARAM_CLAIM_MAX = 3,      /* max queue entries one CTA claims at once (1..1024) [1024] */
-    SSSP_PARAM_L2_PERSIST = 4      /* 1: keep dist[] in a persisting L2 window (raises the
+    SSSP_PARAM_L2_PERSIST = 4,     /* 1: keep dist[] in a persisting L2 window (raises the
                                       device's persisting-L2 limit; never lowers it) [1] */
+    SSSP_PARAM_ADWL = 5,           /* ablation: 1 adaptive thread/warp/CTA bins + hub chunks
+                                      (P:733-780); 0 static thread per vertex [1] */
+    SSSP_PARAM_SYNC = 6            /* ablation: 1 level-synchronous phase 1 (a grid barrier per
+                                      frontier level, the paper's BL); 0 the
+                                      bucket-aware asynchronous phase 1 (BASYN) [0] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

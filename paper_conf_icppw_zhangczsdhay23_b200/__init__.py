@@ -42,6 +42,8 @@ SSSP_PARAM_CTAS_PER_SM = 1
 SSSP_PARAM_SLOT_CAPACITY = 2
 SSSP_PARAM_CLAIM_MAX = 3
 SSSP_PARAM_L2_PERSIST = 4
+SSSP_PARAM_ADWL = 5
+SSSP_PARAM_SYNC = 6
 
 INF_U32 = 0xFFFFFFFF
 
@@ -57,7 +59,7 @@ EXPORTS = (
 class sssp_stats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in (
         "updates", "light_arcs", "heavy_arcs", "vertices_settled", "stale_items", "heavy_vertices",
-        "hub_chunks", "bin_thread", "bin_warp", "bin_cta", "buckets", "rescans", "reachable")] + [
+        "hub_chunks", "bin_thread", "bin_warp", "bin_cta", "buckets", "rescans", "reachable", "levels")] + [
         ("ring_slots", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
         ("run_ms", ctypes.c_float), ("reorder_ms", ctypes.c_float)]
 

@@ -127,7 +127,7 @@ struct __align__(128) Ctl {
   u32 cur, lim, mode, far_min;
   u32 p2_begin, p2_end, err, epochs;
   u32 rescans, rescan_base, changed, sweep_first;
-  u32 sweeps, trace_n, pad1, pad2;
+  u32 sweeps, trace_n, round_end, rounds;  // round_end: level-synchronous mode (ablation)
   u32 pad_a[16];
   u32 bar_count, pad3[31];   // own line: arrivals
   u32 bar_gen, pad4[31];     // own line: spun on
@@ -168,6 +168,8 @@ struct Params {
   float inv_delta;   // f32 graphs: fl32(1/Delta)
   u32 delta_bits;    // light iff wbits < delta_bits
   u32 claim_max;
+  u32 adwl;  // 1: adaptive thread/warp/CTA bins + hub chunks; 0: thread per vertex (ablation)
+  u32 sync;  // 1: level-synchronous phase 1, a grid barrier per frontier level (ablation BL)
 };
 
 constexpr u32 TASK = 32 * UNROLL;  // arcs per warp task
@@ -203,7 +205,7 @@ struct Smem {
   unsigned long long st[ST_N];
   u32 claim_h, claim_n, claim_src;
   // control snapshot
-  u32 mode, cur, lim, p2_begin, p2_end, sweep_first;
+  u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
 };
 
 // ---------------------------------------------------------------- helpers --
@@ -477,7 +479,7 @@ __device__ __forceinline__ u32 batch_item_index(u32 r) {
 // src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
 // phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
 // into the current bucket, hubs stay in the range list).
-template <bool F32, bool PRO, int PH, int N>
+template <bool F32, bool PRO, int PH, int N, bool ADWL = true>
 __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u64 (&it)[N],
                                               const bool (&has)[N], u32 lim, u32 src, u32 slot) {
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
@@ -525,7 +527,13 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
         i64 rb, re;
         item_range<PRO, PH>(p, v, rb, re);
         const i64 l = re - rb;
-        if (l > (i64)HUB_CHUNK && !sweep) {  // hub: ceil(l/4096) chunks any CTA may claim
+        if (!ADWL) {  // ablation: the vertex's own thread walks all its arcs
+          beg[i] = (u32)rb;
+          len[i] = (u32)l;
+          cls[i] = l > 0 ? 3 : 0;
+          c_arcs += (u32)l;
+          c_t += l > 0;
+        } else if (l > (i64)HUB_CHUNK && !sweep) {  // hub: ceil(l/4096) chunks any CTA may claim
           const u32 nc = (u32)((l + HUB_CHUNK - 1) / HUB_CHUNK);
           c_chunks += nc;
           u64* word = (PH == 1) ? &p.sc[slot].word : &p.ctl->hub_word;
@@ -567,6 +575,26 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   for (int i = 0; i < N; ++i)
     if (cls[i]) prefetch_l2(p.arcs + beg[i], len[i] * (u32)sizeof(uint2));
 #endif
+  if (!ADWL) {  // ablation (no ADWL): static thread-per-vertex relaxation
+#pragma unroll 1
+    for (int i = 0; i < N; ++i) {
+      const u32 l = cls[i] == 3 ? len[i] : 0u;
+      const u32 maxl = __reduce_max_sync(SSSP_FULL_MASK, l);
+      for (u32 j0 = 0; j0 < maxl; j0 += UNROLL) {
+        u32 idx[UNROLL], dd[UNROLL];
+        bool valid[UNROLL];
+        uint2 a[UNROLL];
+#pragma unroll
+        for (int k = 0; k < UNROLL; ++k) {
+          valid[k] = j0 + k < l;
+          idx[k] = beg[i] + j0 + k;
+          dd[k] = d[i];
+        }
+        arcs_issue(p, idx, valid, a);
+        relax_finish<F32, PRO, PH>(p, sm, lim, nearb, a, valid, dd);
+      }
+    }
+  }
   // ---- stats (warp-aggregated)
   st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
   if (PH == 1) st_add(sm, ST_STALE, c_stale);
@@ -755,6 +783,13 @@ __device__ void decide(const Params& p, u32 which) {
       return;
     }
     const u32 tail = min((u32)(sc[s].word >> 32), p.cap);
+    if (p.sync && tail > c->round_end) {  // level-synchronous: the next frontier level
+      sc[s].head = c->round_end;
+      c->round_end = tail;
+      c->rounds = c->rounds + 1;
+      c->mode = MODE_PHASE1;
+      return;
+    }
     const u32 b = sc[s].p2;
     c->p2_begin = b;
     c->p2_end = tail;
@@ -770,6 +805,7 @@ __device__ void decide(const Params& p, u32 which) {
       if (fm <= cur) {
         enter_sweep(c);
       } else {
+        c->round_end = min((u32)(sc[s].word >> 32), p.cap);
         c->mode = MODE_PHASE1;
         c->epochs = c->epochs + 1;
       }
@@ -796,6 +832,7 @@ __device__ void decide(const Params& p, u32 which) {
     const u64 lim = (u64)cur + K - 1;  // excludes slot s of bucket cur+K: reset just now
     c->lim = (u32)min(lim, (u64)NONE - 1);
     c->cur = nxt;
+    c->round_end = min((u32)(sc[nxt & p.kmask].word >> 32), p.cap);
     c->mode = MODE_PHASE1;
     c->epochs = c->epochs + 1;
   } else if (which == SYNC_RC) {
@@ -810,6 +847,7 @@ __device__ void decide(const Params& p, u32 which) {
     c->lim = (u32)min((u64)r + K - 1, (u64)NONE - 1);
     c->mode = MODE_RESCAN_FILL;
   } else if (which == SYNC_RF) {
+    c->round_end = min((u32)(sc[c->cur & p.kmask].word >> 32), p.cap);
     c->mode = MODE_PHASE1;
     c->epochs = c->epochs + 1;
     c->rescans = c->rescans + 1;
@@ -871,6 +909,7 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
     sm.p2_begin = vc->p2_begin;
     sm.p2_end = vc->p2_end;
     sm.sweep_first = vc->sweep_first;
+    sm.round_end = vc->round_end;
     sm.st[ST_P_BAR] += (unsigned long long)(clock64() - t_b);
   }
   __syncthreads();
@@ -888,7 +927,13 @@ __device__ void phase1(const Params& p, Smem& sm) {
     if (threadIdx.x == 0) {
       const long long t_c = clock64();
       u32 n = 0, h = 0, ns = 32, waited = 0;
-      for (;;) {
+      if (p.sync) {  // level-synchronous: only this level's entries, all already written
+        const u32 re = sm.round_end;
+        const u32 c = min(max(re / (2 * G), 8u), min(p.claim_max, BATCH));
+        h = ld_relaxed_u32(&sc->head) < re ? atomicAdd(&sc->head, c) : re;
+        n = h < re ? min(c, re - h) : 0u;
+      }
+      for (; !p.sync;) {
         const u64 wv = ld_relaxed_u64(&sc->word);
         const u32 tail = min((u32)(wv >> 32), p.cap);
         if (my_next >= my_end && my_end < p.cap) {
@@ -940,7 +985,10 @@ __device__ void phase1(const Params& p, Smem& sm) {
         it[i] = ld_relaxed_u64(q + h + batch_item_index(i));
       }
     }
-    process_batch<F32, PRO, 1, IPT>(p, sm, it, has, lim, SRC_QUEUE, slot);
+    if (p.adwl)
+      process_batch<F32, PRO, 1, IPT>(p, sm, it, has, lim, SRC_QUEUE, slot);
+    else
+      process_batch<F32, PRO, 1, IPT, false>(p, sm, it, has, lim, SRC_QUEUE, slot);
     if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
   }
 }
@@ -1017,7 +1065,10 @@ __device__ void phase2(const Params& p, Smem& sm) {
       }
       st_relaxed_u64(base_q + batch_item_index(i), SENTINEL);  // recycle the queue entry
     }
-    process_batch<F32, PRO, 2, IPT2>(p, sm, it, has, lim, src, slot);
+    if (p.adwl)
+      process_batch<F32, PRO, 2, IPT2>(p, sm, it, has, lim, src, slot);
+    else
+      process_batch<F32, PRO, 2, IPT2, false>(p, sm, it, has, lim, src, slot);
     if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
   }
 }
@@ -1109,6 +1160,7 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     sm.p2_begin = vc->p2_begin;
     sm.p2_end = vc->p2_end;
     sm.sweep_first = vc->sweep_first;
+    sm.round_end = vc->round_end;
   }
   __syncthreads();
   for (;;) {
@@ -1176,6 +1228,8 @@ __global__ void k_seed(Params p, u32 src) {
     c->hub_word = 0;
     c->hub_head = 0;
     c->trace_n = 0;
+    c->round_end = 1;
+    c->rounds = 0;
   }
 }
 

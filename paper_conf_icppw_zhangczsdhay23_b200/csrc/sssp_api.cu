@@ -72,7 +72,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -276,6 +276,14 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "l2 persist is 0 or 1");
       g->p_l2 = v;
       g->l2_window_bytes = -1;
+      return SSSP_OK;
+    case SSSP_PARAM_ADWL:
+      if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "adwl is 0 or 1");
+      g->p_adwl = v;
+      return SSSP_OK;
+    case SSSP_PARAM_SYNC:
+      if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "sync is 0 or 1");
+      g->p_sync = v;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
@@ -566,6 +574,8 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.inv_delta = dp.inv;
   p.delta_bits = dp.delta_bits;
   p.claim_max = (u32)g->p_claim;
+  p.adwl = (u32)g->p_adwl;
+  p.sync = (u32)g->p_sync;
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal);
@@ -716,6 +726,7 @@ extern "C" sssp_status sssp_get_stats(sssp_graph_t g, sssp_stats* out) {
   out->bin_cta = h[ST_BIN_C];
   out->buckets = c.epochs;
   out->rescans = c.rescans + c.sweeps;
+  out->levels = c.rounds;
   out->reachable = g->have_result ? reach : 0;
   out->ring_slots = g->K_used;
   out->grid_ctas = (u32)g->grid_ctas;

@@ -325,3 +325,26 @@ def test_device_inputs_and_outputs(sssp):
         torch.cuda.synchronize()
         for i, ss in enumerate(srcs):
             assert_same(mat[i].cpu().numpy().view(np.uint32), oracle.dijkstra(g.row, g.col, g.w, int(ss)), "batch")
+
+
+# ------------------------------------------------------- ablation modes ---
+@pytest.mark.parametrize("sync,adwl,flags", [(1, 0, 0), (0, 0, 0), (0, 0, 3), (0, 1, 0), (1, 1, 3)])
+@pytest.mark.parametrize("wt", ["u32", "f32"])
+def test_ablation_modes_parity(sssp, sync, adwl, flags, wt):
+    """BL (sync, static), BASYN, +PRO, +ADWL: every ablation mode is exact."""
+    g = gen.kronecker(12, 16, seed=77, weights=wt)
+    srcs = gen.sample_sources(g, 2, seed=3)
+    delta = 32 if wt == "u32" else 0.1
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if flags:
+            G.reorder(flags)
+        G.set_param(sssp.SSSP_PARAM_SYNC, sync)
+        G.set_param(sssp.SSSP_PARAM_ADWL, adwl)
+        for s in srcs:
+            assert_same(G.sssp(int(s), delta), oracle.dijkstra(g.row, g.col, g.w, int(s)),
+                        f"sync={sync} adwl={adwl} flags={flags} src={s}")
+            st = G.stats()
+            if sync:
+                assert st["levels"] > 0
+            if not adwl:
+                assert st["hub_chunks"] == 0 and st["bin_warp"] == 0 and st["bin_cta"] == 0
