@@ -168,9 +168,13 @@ struct Params {
   float inv_delta;   // f32 graphs: fl32(1/Delta)
   u32 delta_bits;    // light iff wbits < delta_bits
   u32 claim_max;
-  u32 adwl;  // 1: adaptive thread/warp/CTA bins + hub chunks; 0: thread per vertex (ablation)
-  u32 sync;  // 1: level-synchronous phase 1, a grid barrier per frontier level (ablation BL)
+  // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
+  // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL).
+  // Params stays <= 128 bytes: larger, it spills around the out-of-line pb_flush call.
+  u32 flags;
 };
+
+static_assert(sizeof(Params) <= 128, "Params > 128 B spills around the out-of-line pb_flush call");
 
 constexpr u32 TASK = 32 * UNROLL;  // arcs per warp task
 constexpr u32 BATCH = DS_THREADS * IPT;        // queue items per phase-1 CTA batch
@@ -783,7 +787,7 @@ __device__ void decide(const Params& p, u32 which) {
       return;
     }
     const u32 tail = min((u32)(sc[s].word >> 32), p.cap);
-    if (p.sync && tail > c->round_end) {  // level-synchronous: the next frontier level
+    if ((p.flags & 2u) && tail > c->round_end) {  // level-synchronous: the next frontier level
       sc[s].head = c->round_end;
       c->round_end = tail;
       c->rounds = c->rounds + 1;
@@ -916,7 +920,7 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
 }
 
 // ------------------------------------------------------------ phases ------
-template <bool F32, bool PRO>
+template <bool F32, bool PRO, bool ABL>
 __device__ void phase1(const Params& p, Smem& sm) {
   const u32 slot = sm.cur & p.kmask, lim = sm.lim;
   SlotCtl* sc = p.sc + slot;
@@ -927,13 +931,13 @@ __device__ void phase1(const Params& p, Smem& sm) {
     if (threadIdx.x == 0) {
       const long long t_c = clock64();
       u32 n = 0, h = 0, ns = 32, waited = 0;
-      if (p.sync) {  // level-synchronous: only this level's entries, all already written
+      if (ABL && (p.flags & 2u)) {  // level-synchronous: only this level's entries, all already written
         const u32 re = sm.round_end;
         const u32 c = min(max(re / (2 * G), 8u), min(p.claim_max, BATCH));
         h = ld_relaxed_u32(&sc->head) < re ? atomicAdd(&sc->head, c) : re;
         n = h < re ? min(c, re - h) : 0u;
       }
-      for (; !p.sync;) {
+      for (; !(ABL && (p.flags & 2u));) {
         const u64 wv = ld_relaxed_u64(&sc->word);
         const u32 tail = min((u32)(wv >> 32), p.cap);
         if (my_next >= my_end && my_end < p.cap) {
@@ -985,15 +989,15 @@ __device__ void phase1(const Params& p, Smem& sm) {
         it[i] = ld_relaxed_u64(q + h + batch_item_index(i));
       }
     }
-    if (p.adwl)
+    if (!ABL || (p.flags & 1u))
       process_batch<F32, PRO, 1, IPT>(p, sm, it, has, lim, SRC_QUEUE, slot);
     else
-      process_batch<F32, PRO, 1, IPT, false>(p, sm, it, has, lim, SRC_QUEUE, slot);
+      process_batch<F32, PRO, 1, IPT, !ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
     if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
   }
 }
 
-template <bool F32, bool PRO>
+template <bool F32, bool PRO, bool ABL>
 __device__ void phase2(const Params& p, Smem& sm) {
   const u32 slot = sm.cur & p.kmask, lim = sm.lim;
   u64* q = p.items + (u64)slot * p.cap;
@@ -1065,10 +1069,10 @@ __device__ void phase2(const Params& p, Smem& sm) {
       }
       st_relaxed_u64(base_q + batch_item_index(i), SENTINEL);  // recycle the queue entry
     }
-    if (p.adwl)
+    if (!ABL || (p.flags & 1u))
       process_batch<F32, PRO, 2, IPT2>(p, sm, it, has, lim, src, slot);
     else
-      process_batch<F32, PRO, 2, IPT2, false>(p, sm, it, has, lim, src, slot);
+      process_batch<F32, PRO, 2, IPT2, !ABL>(p, sm, it, has, lim, src, slot);
     if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
   }
 }
@@ -1142,7 +1146,9 @@ __device__ void sweep(const Params& p, Smem& sm) {
   }
 }
 
-template <bool F32, bool PRO>
+// ABL = ablation build (SSSP_PARAM_ADWL = 0 / SSSP_PARAM_SYNC = 1 paths compiled in);
+// the default kernel (ABL = false) carries none of that code.
+template <bool F32, bool PRO, bool ABL>
 __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) {
   __shared__ Smem sm;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -1167,10 +1173,10 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     const u32 mode = sm.mode;
     if (mode == MODE_DONE) break;
     if (mode == MODE_PHASE1) {
-      phase1<F32, PRO>(p, sm);
+      phase1<F32, PRO, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_P1);
     } else if (mode == MODE_PHASE2) {
-      phase2<F32, PRO>(p, sm);
+      phase2<F32, PRO, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (mode == MODE_RESCAN_CLEAR) {
       rescan_clear(p);

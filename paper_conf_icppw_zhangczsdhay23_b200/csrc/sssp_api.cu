@@ -495,9 +495,13 @@ static sssp_status ensure_run_buffers(sssp_graph_t g, u32 K, u32 cap) {
 }
 
 typedef void (*ds_kernel_t)(Params);
-static ds_kernel_t pick_kernel(bool f32, bool pro) {
-  if (f32) return pro ? k_delta_step<true, true> : k_delta_step<true, false>;
-  return pro ? k_delta_step<false, true> : k_delta_step<false, false>;
+static ds_kernel_t pick_kernel(bool f32, bool pro, bool abl) {
+  if (abl) {
+    if (f32) return pro ? k_delta_step<true, true, true> : k_delta_step<true, false, true>;
+    return pro ? k_delta_step<false, true, true> : k_delta_step<false, false, true>;
+  }
+  if (f32) return pro ? k_delta_step<true, true, false> : k_delta_step<true, false, false>;
+  return pro ? k_delta_step<false, true, false> : k_delta_step<false, false, false>;
 }
 
 static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParams& dp, bool timed) {
@@ -548,7 +552,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
     }
     cudaGetLastError();
   }
-  ds_kernel_t kern = pick_kernel(f32, pro);
+  ds_kernel_t kern = pick_kernel(f32, pro, g->p_adwl == 0 || g->p_sync != 0);
   int per_sm = 0;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, DS_THREADS, 0));
   if (per_sm < 1) return fail(SSSP_ERR_INTERNAL, "persistent kernel cannot be resident");
@@ -574,8 +578,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.inv_delta = dp.inv;
   p.delta_bits = dp.delta_bits;
   p.claim_max = (u32)g->p_claim;
-  p.adwl = (u32)g->p_adwl;
-  p.sync = (u32)g->p_sync;
+  p.flags = (g->p_adwl ? 1u : 0u) | (g->p_sync ? 2u : 0u);
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal);
