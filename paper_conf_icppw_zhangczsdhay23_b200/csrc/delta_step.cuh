@@ -298,8 +298,28 @@ __device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
 // distinct bucket queue (tail and pend in one atomicAdd). Entries beyond the
 // ring horizon or a full queue are dropped and recorded in far_min. In the
 // sweep fall-back (nearb != NONE) entries of bucket nearb mark xd[] instead.
+// What pb_flush needs, passed by value (48 B) to the out-of-line call.
+struct FlushCtx {
+  SlotCtl* sc;
+  u64* items;
+  Ctl* ctl;
+  u32* xd;
+  u32 cap, kmask, delta_u;
+  float inv_delta;
+};
+
 template <bool F32>
-__device__ __noinline__ void pb_flush(const Params p, Smem& sm, u32 lim, u32 nearb) {
+__device__ __forceinline__ u32 bucket_of_f(const FlushCtx& p, u32 d) {
+  if (F32) {
+    u32 b = __float2uint_rz(__fmul_rn(__uint_as_float(d), p.inv_delta));
+    return b >= NONE ? NONE - 1 : b;
+  } else {
+    return d / p.delta_u;
+  }
+}
+
+template <bool F32>
+__device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, u32 nearb) {
   const u32 lane = lane_id(), w = threadIdx.x >> 5;
   const u32 n = sm.pb_n[w];
   if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)n);
@@ -308,7 +328,7 @@ __device__ __noinline__ void pb_flush(const Params p, Smem& sm, u32 lim, u32 nea
     bool ok = i < n;
     const u64 e = ok ? sm.pb[w][i] : 0ULL;
     const u32 v = (u32)e, nd = (u32)(e >> 32);
-    const u32 x = ok ? bucket_of<F32>(p, nd) : 0u;
+    const u32 x = ok ? bucket_of_f<F32>(p, nd) : 0u;
     if (ok && x == nearb) {
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
@@ -339,6 +359,12 @@ __device__ __noinline__ void pb_flush(const Params p, Smem& sm, u32 lim, u32 nea
   __syncwarp();
   if (lane == 0) sm.pb_n[w] = 0;
   __syncwarp();
+}
+
+template <bool F32>
+__device__ __forceinline__ void pb_flush(const Params& p, Smem& sm, u32 lim, u32 nearb) {
+  const FlushCtx f = {p.sc, p.items, p.ctl, p.xd, p.cap, p.kmask, p.delta_u, p.inv_delta};
+  pb_flush_impl<F32>(f, sm, lim, nearb);
 }
 
 // Stage up to UNROLL pushes per lane into the warp's buffer (all 32 lanes).
