@@ -211,12 +211,19 @@ def main():
 
     import torch
 
+    # SSSP_DIST_BACKEND=gloo (test only): exercise the multi-rank logic with
+    # several ranks sharing fewer GPUs; the product path is NCCL, one GPU per rank.
+    backend = os.environ.get("SSSP_DIST_BACKEND", "nccl")
+    dev = (local % torch.cuda.device_count()) if world > 1 else 0
     if world > 1:
         import torch.distributed as dist
 
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = local if world > 1 else 0
+        torch.cuda.set_device(dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
+    tdev = f"cuda:{dev}" if backend == "nccl" else "cpu"
     torch.cuda.set_device(dev)
     import paper_conf_icppw_zhangczsdhay23_b200 as sssp
 
@@ -261,7 +268,7 @@ def main():
     t_ms = ev0.elapsed_time(ev1)
     kt_total, kt_n = G.kernel_time(reset=True)
     if world > 1:
-        tt = torch.tensor([t_ms], device=f"cuda:{dev}")
+        tt = torch.tensor([t_ms], device=tdev)
         torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
         torch.distributed.barrier()
         t_ms = float(tt.item())
@@ -284,7 +291,7 @@ def main():
             if rank == 0:
                 pinned.copy_(rows.view(torch.int32) if rows.dtype != torch.int32 else rows)
         torch.distributed.barrier()
-        te = torch.tensor([time.perf_counter() - t0], device=f"cuda:{dev}")
+        te = torch.tensor([time.perf_counter() - t0], device=tdev)
         torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
         e2e_multi = {"value": round(world * ne * g.m / float(te.item()) / 1e9, 4), "unit": "GTEPS",
                      "h2d_bytes_per_step": 8 * world, "d2h_bytes_per_step": 4 * g.V * world,

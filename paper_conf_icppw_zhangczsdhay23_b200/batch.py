@@ -44,6 +44,8 @@ def gather_rows(local_rows, n_sources: int, dst: int = 0, group=None):
         pad = torch.zeros((k - local_rows.shape[0], V), dtype=local_rows.dtype, device=local_rows.device)
         local_rows = torch.cat([local_rows, pad], 0)
     local_rows = local_rows.contiguous()
+    if dist.get_backend(group) != "nccl" and local_rows.is_cuda:  # gloo: host staging (tests)
+        local_rows = local_rows.cpu()
     bufs = [torch.empty_like(local_rows) for _ in range(world)] if rank == dst else None
     dist.gather(local_rows, bufs, dst=dst, group=group)
     if rank != dst:
