@@ -17,12 +17,14 @@ def main():
     ap.add_argument("--config", default="C4")
     ap.add_argument("--runs", type=int, default=8)
     ap.add_argument("--rounds", type=int, default=3)
+    ap.add_argument("--deltas", type=float, nargs="*", default=None)
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     import torch  # noqa: F401  (CUDA context)
 
     g = gen.make_config(a.config)
     delta = gen.CONFIGS[a.config]["delta"]
+    deltas = a.deltas or [delta]
     srcs = gen.sample_sources(g, a.runs, seed=7)
     P, I64, I, D = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_double
     handles = []
@@ -41,17 +43,17 @@ def main():
         t, n = ctypes.c_double(), ctypes.c_int64()
         L.sssp_kernel_time(h, ctypes.byref(t), ctypes.byref(n), 1)
         handles.append((path, L, h))
-    res = {p: [] for p in a.libs}
+    res = {(p, d): [] for p in a.libs for d in deltas}
     for r in range(a.rounds):
         for path, L, h in handles:
-            for s in srcs:
-                assert L.sssp_run(h, int(s), float(delta)) == 0
-            t, n = ctypes.c_double(), ctypes.c_int64()
-            L.sssp_kernel_time(h, ctypes.byref(t), ctypes.byref(n), 1)
-            res[path].append(t.value / n.value)
-    for path in a.libs:
-        v = res[path]
-        print(f"{os.path.basename(path):24s} mean/round ms: " + " ".join(f"{x:.3f}" for x in v)
+            for d in deltas:
+                for s in srcs:
+                    assert L.sssp_run(h, int(s), float(d)) == 0
+                t, n = ctypes.c_double(), ctypes.c_int64()
+                L.sssp_kernel_time(h, ctypes.byref(t), ctypes.byref(n), 1)
+                res[(path, d)].append(t.value / n.value)
+    for (path, d), v in res.items():
+        print(f"{os.path.basename(path):20s} delta={d:<8g} mean/round ms: " + " ".join(f"{x:.3f}" for x in v)
               + f"  | best {min(v):.3f}")
 
 
