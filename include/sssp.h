@@ -91,7 +91,10 @@ sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta);
 
 /* Copy the last run's distances (V elements of the graph's weight type, in
  * ORIGINAL vertex order; unreachable = 0xFFFFFFFF for u32, +inf for f32) to
- * `out` (host or device per `where`). HOST synchronises the stream.
+ * `out` (host or device per `where`). HOST synchronises the stream; a pinned,
+ * device-mapped host buffer (cudaHostAlloc, torch pin_memory) is written
+ * directly by the output gather kernel, pageable memory is staged through a
+ * library-owned device buffer (allocated on first use, freed by destroy).
  * SSSP_ERR_INVALID_STATE if no successful run since create/reorder;
  * SSSP_ERR_OVERFLOW if a u32 distance overflowed during the run. */
 sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory where);

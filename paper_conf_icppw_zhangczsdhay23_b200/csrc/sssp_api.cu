@@ -56,6 +56,7 @@ struct sssp_graph_s {
   SlotCtl* sc = nullptr;
   u64* items = nullptr;
   u64* hub_items = nullptr;
+  u32* out_tmp = nullptr;  // [V] staging for sssp_distances into pageable host memory
   unsigned long long* stats = nullptr;
   TraceEnt* trace = nullptr;
   u32 K_alloc = 0, cap_alloc = 0, hub_cap = 0;
@@ -218,7 +219,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
   void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
-                  g->items, g->hub_items, g->stats, g->trace};
+                  g->items, g->hub_items, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& e : g->ev)
@@ -664,14 +665,25 @@ extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory whe
   DeviceGuard dg(g->device);
   cudaStream_t s = g->stream;
   u32* dst = (u32*)out;
-  u32* tmp = nullptr;
-  if (where == SSSP_MEM_HOST) CU(cudaMallocAsync(&tmp, sizeof(u32) * g->V, s));
-  k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, tmp ? tmp : dst);
-  CU(cudaGetLastError());
-  if (tmp) {
-    CU(cudaMemcpyAsync(dst, tmp, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
-    CU(cudaFreeAsync(tmp, s));
+  bool staged = false;
+  if (where == SSSP_MEM_HOST) {
+    // Pinned, device-mapped host memory (cudaHostAlloc / torch pin_memory) is
+    // written directly by the output gather over the host link: a8 fused with
+    // the D2H copy. Pageable memory goes through a persistent device staging
+    // buffer and one cudaMemcpyAsync (no per-call allocation).
+    cudaPointerAttributes pa;
+    if (cudaPointerGetAttributes(&pa, out) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+        pa.devicePointer != nullptr) {
+      dst = (u32*)pa.devicePointer;
+    } else {
+      cudaGetLastError();
+      if (!g->out_tmp) CU(cudaMalloc(&g->out_tmp, sizeof(u32) * g->V));
+      staged = true;
+    }
   }
+  k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, staged ? g->out_tmp : dst);
+  CU(cudaGetLastError());
+  if (staged) CU(cudaMemcpyAsync(out, g->out_tmp, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
   return check_run_errors(g);
 }
 

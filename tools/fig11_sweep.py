@@ -1,0 +1,77 @@
+"""NEXT-3: the paper's Fig. 11 sweep on one B200.
+
+Kronecker SCALE 22/23/24 x edgefactor 8/16/32/64 (Graph500 A=.57 B=.19 C=.19
+D=.05, scrambled, symmetrised), u32 weights U{1..1000} (the paper's stated
+weight range), PRO on. Per graph: a short Delta sweep on 4
+sources, then GTEPS = m / t (m = EF * 2^SCALE input edges) as
+the mean over N seeded sources at the best Delta, persistent-kernel time
+from CUDA events (sssp_kernel_time). Prints one line per graph plus the
+paper's V100 number.
+
+python tools/fig11_sweep.py [--scales 22 23 24] [--efs 8 16 32 64] [--sources 16]
+"""
+import argparse
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+PAPER = {  # Fig. 11 V100 GTEPS
+    (22, 8): 8.81, (22, 16): 16.78, (22, 32): 21.26, (22, 64): 35.35,
+    (23, 8): 9.32, (23, 16): 20.60, (23, 32): 23.65, (23, 64): 38.98,
+    (24, 8): 11.28, (24, 16): 20.16, (24, 32): 26.23, (24, 64): 40.09,
+}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--scales", type=int, nargs="*", default=[22, 23, 24])
+    ap.add_argument("--efs", type=int, nargs="*", default=[8, 16, 32, 64])
+    ap.add_argument("--deltas", type=float, nargs="*", default=[80, 160, 320])
+    ap.add_argument("--sources", type=int, default=16)
+    ap.add_argument("--seed", type=int, default=11)
+    a = ap.parse_args()
+    import torch  # noqa: F401  (CUDA context, device memory)
+
+    import paper_conf_icppw_zhangczsdhay23_b200 as sssp
+
+    print("scale ef  V          arcs        best_delta  ms/SSSP  GTEPS   paper_V100  ratio  gen_s  reorder_ms", flush=True)
+    for s in a.scales:
+        for ef in a.efs:
+            t0 = time.time()
+            g = gen.kronecker(s, ef, seed=a.seed, weights="u32", lo=1, hi=1000)
+            gen_s = time.time() - t0
+            srcs = gen.sample_sources(g, a.sources, seed=7)
+            with sssp.Graph(g.row, g.col, g.w, device=0) as G:
+                G.reorder()
+                reorder_ms = G.stats()["reorder_ms"]
+                best = None
+                for d in a.deltas:
+                    G.run(int(srcs[0]), d)  # warm-up (heavy offsets for this Delta)
+                    G.kernel_time(reset=True)
+                    for x in srcs[:4]:
+                        G.run(int(x), d)
+                    t, n = G.kernel_time(reset=True)
+                    if best is None or t / n < best[1]:
+                        best = (d, t / n)
+                d = best[0]
+                G.run(int(srcs[0]), d)
+                G.kernel_time(reset=True)
+                for x in srcs:
+                    G.run(int(x), d)
+                t, n = G.kernel_time(reset=True)
+                ms = t / n
+            m = ef * (1 << s)
+            gteps = m / (ms * 1e-3) / 1e9
+            p = PAPER.get((s, ef))
+            print(f"{s:5d} {ef:3d} {g.V:<10d} {g.A:<11d} {d:<11g} {ms:8.3f} {gteps:7.2f} {p!s:>10} "
+                  f"{gteps / p if p else float('nan'):6.2f} {gen_s:6.1f} {reorder_ms:9.1f}", flush=True)
+            del g
+
+
+if __name__ == "__main__":
+    main()
