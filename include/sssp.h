@@ -160,9 +160,13 @@ typedef enum {
                                       device's persisting-L2 limit; never lowers it) [1] */
     SSSP_PARAM_ADWL = 5,           /* ablation: 1 adaptive thread/warp/CTA bins + hub chunks
                                       (P:733-780); 0 static thread per vertex [1] */
-    SSSP_PARAM_SYNC = 6            /* ablation: 1 level-synchronous phase 1 (a grid barrier per
+    SSSP_PARAM_SYNC = 6,           /* ablation: 1 level-synchronous phase 1 (a grid barrier per
                                       frontier level, the paper's BL); 0 the
                                       bucket-aware asynchronous phase 1 (BASYN) [0] */
+    SSSP_PARAM_P2_EDGE_BALANCED = 7 /* phases 2&3 with equal heavy arcs per warp
+                                      for buckets with >= value settled entries; smaller
+                                      buckets (and -1 = never) relax heavy arcs through the
+                                      phase-1 vertex bins [-1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

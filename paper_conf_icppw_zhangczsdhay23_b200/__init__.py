@@ -44,6 +44,7 @@ SSSP_PARAM_CLAIM_MAX = 3
 SSSP_PARAM_L2_PERSIST = 4
 SSSP_PARAM_ADWL = 5
 SSSP_PARAM_SYNC = 6
+SSSP_PARAM_P2_EDGE_BALANCED = 7
 
 INF_U32 = 0xFFFFFFFF
 

@@ -82,10 +82,12 @@ enum : u32 {
   MODE_RESCAN_CLEAR = 3,
   MODE_RESCAN_FILL = 4,
   MODE_SWEEP_LIGHT = 5,
-  MODE_SWEEP_HEAVY = 6
+  MODE_SWEEP_HEAVY = 6,
+  MODE_P2_COMPACT = 7,  // edge-balanced phase 2, step 1: settled entries -> heavy-arc offsets
+  MODE_P2_RELAX = 8     // ... step 2: equal heavy-arc ranges per warp
 };
 enum : u32 { ERR_OVERFLOW = 1, ERR_INTERNAL = 2 };
-enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5 };
+enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5, SYNC_P2C = 6 };
 enum : u32 { SRC_QUEUE = 0, SRC_STATIC = 1, SRC_HUB = 2, SRC_SWEEP = 3 };
 
 enum {
@@ -132,7 +134,8 @@ struct __align__(128) Ctl {
   u32 bar_count, pad3[31];   // own line: arrivals
   u32 bar_gen, pad4[31];     // own line: spun on
   u32 p2_head, pad5[31];     // own line: phase-2 static tickets
-  u64 hub_word;              // phase-2 chunk queue: (tail << 32) | pend
+  u64 hub_word;              // phase-2 chunk queue: (tail << 32) | pend; edge-balanced
+                             // phase 2: (compacted entries << 32) | heavy arcs
   u32 hub_head, pad6[29];
 };
 
@@ -163,13 +166,16 @@ struct Params {
   u64* hub_items;         // [hub_cap]
   unsigned long long* stats;  // [ST_N]
   TraceEnt* trace;            // [TRACE_CAP] barrier timeline of the last run
+  u32* p2o;  // [cap] edge-balanced phase 2: first heavy-arc rank of each compacted entry,
+             // followed by uint2 [cap] {arc index - rank, d} (see p2_compact)
   u32 V, K, kmask, cap, hub_cap;
   u32 delta_u;       // u32 graphs: integer Delta >= 1
   float inv_delta;   // f32 graphs: fl32(1/Delta)
   u32 delta_bits;    // light iff wbits < delta_bits
   u32 claim_max;
   // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
-  // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL).
+  // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL;
+  // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries).
   // Params stays <= 128 bytes: larger, it spills around the out-of-line pb_flush call.
   u32 flags;
 };
@@ -806,6 +812,13 @@ __device__ void decide(const Params& p, u32 which) {
   volatile Ctl* c = p.ctl;
   volatile SlotCtl* sc = p.sc;
   const u32 K = p.K;
+  if (which == SYNC_P2C) {  // entries compacted: relax their heavy arcs, if any
+    if ((u32)c->hub_word != 0) {
+      c->mode = MODE_P2_RELAX;
+      return;
+    }
+    which = SYNC_P2;
+  }
   if (which == SYNC_P1) {
     const u32 cur = c->cur, s = cur & p.kmask;
     if (c->far_min <= cur) {  // phase-1 work was dropped (queue full)
@@ -823,6 +836,12 @@ __device__ void decide(const Params& p, u32 which) {
     const u32 b = sc[s].p2;
     c->p2_begin = b;
     c->p2_end = tail;
+    if ((p.flags & 4u) && tail - b >= (p.flags >> 8)) {  // edge-balanced phase 2
+      c->hub_word = 0;
+      c->p2_head = 0;
+      c->mode = MODE_P2_COMPACT;
+      return;
+    }
     c->p2_head = b;
     c->hub_word = (u64)(tail - b);  // pending = static entries; chunks add to it
     c->hub_head = 0;
@@ -1103,6 +1122,204 @@ __device__ void phase2(const Params& p, Smem& sm) {
   }
 }
 
+// ------------------------------------------- edge-balanced phase 2 -------
+// The paper's phases 2&3 kernel gives every thread the same number of heavy
+// edges (static load balancing). Here: (1) p2_compact turns the
+// bucket's settled range [p2_begin, p2_end) into a dense list of the entries
+// that are final (d == dist[v], Alg. 2 l.14) and have heavy arcs, each with
+// the rank of its first heavy arc (one 64-bit atomicAdd per CTA batch hands
+// out (entry, arc-rank) bases together, so ranks grow with the list index);
+// (2) after a grid barrier, p2_relax splits the rank range [0, T) into
+// equal-arc pieces claimed by warps. A warp maps arc rank x to its owner entry
+// (the last entry with rank <= x) with a 32-entry window held in registers
+// (one coalesced load per 31 entries, shuffle binary search per arc), so hubs
+// and small vertices are spread over warps by arcs, not by vertices.
+// Measured on B200 (profiles/r01c): no faster than the vertex-bin phase 2 on
+// C4 and 15 % slower on C3, so it is off by default (SSSP_PARAM_P2_EDGE_BALANCED).
+template <bool F32, bool PRO>
+__device__ void p2_compact(const Params& p, Smem& sm) {
+  const u32 slot = sm.cur & p.kmask;
+  u64* q = p.items + (u64)slot * p.cap;
+  const u32 b0 = sm.p2_begin, b1 = sm.p2_end;
+  uint2* sd = reinterpret_cast<uint2*>(p.p2o + ((p.cap + 1) & ~1u));
+  const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  constexpr u32 CB = DS_THREADS * IPT2;
+  u32 c_live = 0, c_arcs = 0;
+  for (u32 base = b0 + blockIdx.x * CB; base < b1; base += gridDim.x * CB) {
+    u64 e[IPT2];
+    bool has[IPT2];
+#pragma unroll
+    for (int i = 0; i < IPT2; ++i) {
+      const u32 pos = base + i * DS_THREADS + tid;
+      has[i] = pos < b1;
+      e[i] = has[i] ? ld_relaxed_u64(q + pos) : SENTINEL;
+    }
+    u32 cd[IPT2];
+#pragma unroll
+    for (int i = 0; i < IPT2; ++i) {
+      if (has[i]) st_relaxed_u64(q + base + i * DS_THREADS + tid, SENTINEL);  // recycle
+      has[i] = has[i] && !((u32)e[i] & CHUNK_FLAG);  // phase-1 hub chunks: no vertex
+      cd[i] = has[i] ? ld_cg(p.dist + (u32)e[i]) : 0u;
+    }
+    u32 hl[IPT2], st[IPT2];
+    u64 x = 0;
+#pragma unroll
+    for (int i = 0; i < IPT2; ++i) {
+      hl[i] = 0;
+      st[i] = 0;
+      if (has[i] && (u32)(e[i] >> 32) == cd[i]) {  // final in this bucket
+        const u32 v = (u32)e[i];
+        const uint2 r = p.rowc[v];
+        st[i] = PRO ? r.y : r.x;
+        hl[i] = p.rowc[v + 1].x - st[i];
+        ++c_live;
+        c_arcs += hl[i];
+        if (hl[i]) x += (1ULL << 32) | hl[i];
+      }
+    }
+    u64 tot;
+    u64 pre = warp_exclusive_scan(x, &tot);
+    if (lane == 31) sm.scan_ws[w] = tot;
+    __syncthreads();
+    u64 acc = 0, all = 0;
+#pragma unroll
+    for (int i = 0; i < DS_WARPS; ++i) {
+      const u64 sv = sm.scan_ws[i];
+      if (i < (int)w) acc += sv;
+      all += sv;
+    }
+    if (tid == 0 && all) {
+      const u64 g = atomicAdd(&p.ctl->hub_word, all);
+      sm.claim_h = (u32)(g >> 32);
+      sm.claim_n = (u32)g;
+    }
+    __syncthreads();
+    if (all) {
+      pre += acc;
+      u32 idx = sm.claim_h + (u32)(pre >> 32), rank = sm.claim_n + (u32)pre;
+#pragma unroll
+      for (int i = 0; i < IPT2; ++i) {
+        if (hl[i]) {
+          p.p2o[idx] = rank;
+          sd[idx] = make_uint2(st[i] - rank, (u32)(e[i] >> 32));  // arc index = rank + .x
+          ++idx;
+          rank += hl[i];
+        }
+      }
+    }
+    __syncthreads();  // scan_ws / claim_* reused by the next batch
+  }
+  st_add(sm, ST_HEAVYV, c_live);
+  st_add(sm, ST_HEAVY, c_arcs);
+}
+
+template <bool F32, bool PRO>
+__device__ void p2_relax(const Params& p, Smem& sm) {
+  const u64 hw = ld_relaxed_u64(&p.ctl->hub_word);
+  const u32 n = (u32)(hw >> 32), T = (u32)hw;
+  const u32 lane = lane_id(), lim = sm.lim;
+  const u32* O = p.p2o;
+  const uint2* sd = reinterpret_cast<const uint2*>(p.p2o + ((p.cap + 1) & ~1u));
+  const u32 W = gridDim.x * DS_WARPS;
+  u32* head = &p.ctl->p2_head;
+  // window over entries [wb, wb+32): rank, {arc index - rank, d}; NONE past n
+  u32 wb = 0, wv = NONE, wx = 0, wy = 0;
+  auto load_window = [&]() {
+    const u32 j = wb + lane;
+    wv = NONE;
+    if (j < n) {
+      wv = ld_cg(O + j);
+      const uint2 t = __ldcg(sd + j);
+      wx = t.x;
+      wy = t.y;
+    }
+  };
+  auto setup = [&](u32 tb, u32 ce, u32(&idx)[UNROLL], bool(&valid)[UNROLL], u32(&dd)[UNROLL]) {
+    bool pend[UNROLL];
+#pragma unroll
+    for (int k = 0; k < UNROLL; ++k) {
+      const u32 xk = tb + k * 32 + lane;
+      valid[k] = tb < ce && xk < ce;
+      pend[k] = valid[k];
+      idx[k] = 0;
+      dd[k] = 0;
+    }
+    for (;;) {
+      const u32 wlast = __shfl_sync(SSSP_FULL_MASK, wv, 31);
+      bool left = false;
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        const u32 xk = tb + k * 32 + lane;
+        u32 j = 0;  // last window entry with rank <= xk (entry 0 always qualifies)
+#pragma unroll
+        for (u32 s = 16; s; s >>= 1) {
+          const u32 t = __shfl_sync(SSSP_FULL_MASK, wv, j + s);
+          if (t <= xk) j += s;
+        }
+        const u32 ax = __shfl_sync(SSSP_FULL_MASK, wx, j);
+        const u32 ay = __shfl_sync(SSSP_FULL_MASK, wy, j);
+        if (pend[k] && xk < wlast) {
+          idx[k] = xk + ax;
+          dd[k] = ay;
+          pend[k] = false;
+        }
+        left |= pend[k];
+      }
+      if (!__any_sync(SSSP_FULL_MASK, left)) break;
+      wb += 31;  // every pending rank is >= the window's last rank
+      load_window();
+    }
+  };
+  for (;;) {
+    u32 c0 = 0, cl = 0;
+    if (lane == 0) {
+      const u32 seen = ld_relaxed_u32(head);
+      const u32 rem = seen < T ? T - seen : 0u;
+      cl = min(max((rem / (2 * W)) & ~(TASK - 1), 8 * TASK), 64 * TASK);  // guided self-scheduling
+      c0 = atomicAdd(head, cl);
+    }
+    c0 = __shfl_sync(SSSP_FULL_MASK, c0, 0);
+    cl = __shfl_sync(SSSP_FULL_MASK, cl, 0);
+    if (c0 >= T) break;
+    const u32 ce = min(c0 + cl, T);
+    // owner of c0: 32-ary search over the ranks
+    u32 lo = 0, hi = n;
+    while (hi - lo > 32) {
+      const u32 step = (hi - lo + 31) / 32;
+      const u32 j = lo + lane * step;
+      const u32 v = j < hi ? ld_cg(O + j) : NONE;
+      const u32 m = __ballot_sync(SSSP_FULL_MASK, v <= c0);
+      lo += (31 - __clz(m)) * step;
+      hi = min(lo + step, hi);
+    }
+    wb = lo;
+    load_window();
+    u32 idx[UNROLL], dd[UNROLL];
+    bool valid[UNROLL];
+    uint2 a[UNROLL];
+    u32 tb = c0;
+    setup(tb, ce, idx, valid, dd);
+    arcs_issue(p, idx, valid, a);
+    while (tb < ce) {
+      const u32 tb2 = tb + TASK;
+      u32 idx2[UNROLL], dd2[UNROLL];
+      bool valid2[UNROLL];
+      uint2 a2[UNROLL];
+      setup(tb2, ce, idx2, valid2, dd2);
+      arcs_issue(p, idx2, valid2, a2);  // next task's arcs in flight ...
+      relax_finish<F32, PRO, 2>(p, sm, lim, NONE, a, valid, dd);  // ... while this one completes
+      tb = tb2;
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        a[k] = a2[k];
+        valid[k] = valid2[k];
+        dd[k] = dd2[k];
+      }
+    }
+  }
+  if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
+}
+
 // Rescan stage 1: clear every queue entry still holding a value.
 __device__ void rescan_clear(const Params& p) {
   const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1203,6 +1420,12 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
       grid_barrier(p, sm, SYNC_P1);
     } else if (mode == MODE_PHASE2) {
       phase2<F32, PRO, ABL>(p, sm);
+      grid_barrier(p, sm, SYNC_P2);
+    } else if (mode == MODE_P2_COMPACT) {
+      p2_compact<F32, PRO>(p, sm);
+      grid_barrier(p, sm, SYNC_P2C);
+    } else if (mode == MODE_P2_RELAX) {
+      p2_relax<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (mode == MODE_RESCAN_CLEAR) {
       rescan_clear(p);

@@ -56,6 +56,7 @@ struct sssp_graph_s {
   SlotCtl* sc = nullptr;
   u64* items = nullptr;
   u64* hub_items = nullptr;
+  u32* p2o = nullptr;  // [cap] + uint2 [cap]: edge-balanced phase-2 scratch
   u32* out_tmp = nullptr;  // [V] staging for sssp_distances into pageable host memory
   unsigned long long* stats = nullptr;
   TraceEnt* trace = nullptr;
@@ -73,7 +74,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -219,7 +220,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
   void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
-                  g->items, g->hub_items, g->stats, g->trace, g->out_tmp};
+                  g->items, g->hub_items, g->p2o, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& e : g->ev)
@@ -285,6 +286,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_SYNC:
       if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "sync is 0 or 1");
       g->p_sync = v;
+      return SSSP_OK;
+    case SSSP_PARAM_P2_EDGE_BALANCED:
+      if (v < -1 || v > 0xFFFFFF) return fail(SSSP_ERR_INVALID_ARGUMENT, "p2 edge-balanced threshold in [-1, 2^24)");
+      g->p_p2eb = v;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
@@ -473,9 +478,12 @@ static sssp_status ensure_run_buffers(sssp_graph_t g, u32 K, u32 cap) {
   if (K > g->K_alloc || cap != g->cap_alloc) {
     if (g->items) CU(cudaFree(g->items));
     if (g->sc) CU(cudaFree(g->sc));
+    if (g->p2o) CU(cudaFree(g->p2o));
     g->items = nullptr;
     g->sc = nullptr;
+    g->p2o = nullptr;
     CU(cudaMalloc(&g->items, sizeof(u64) * (size_t)K * cap));
+    CU(cudaMalloc(&g->p2o, sizeof(u32) * (((size_t)cap + 1) & ~(size_t)1) + sizeof(uint2) * (size_t)cap));
     CU(cudaMalloc(&g->sc, sizeof(SlotCtl) * K));
     CU(cudaMemsetAsync(g->sc, 0, sizeof(SlotCtl) * K, s));
     g->K_alloc = K;
@@ -579,7 +587,10 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.inv_delta = dp.inv;
   p.delta_bits = dp.delta_bits;
   p.claim_max = (u32)g->p_claim;
+  p.p2o = g->p2o;
   p.flags = (g->p_adwl ? 1u : 0u) | (g->p_sync ? 2u : 0u);
+  // edge-balanced phase 2 (not in the static thread-per-vertex ablation)
+  if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal);

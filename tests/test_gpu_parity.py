@@ -166,6 +166,7 @@ def test_hub_chunks(sssp):
         exp = oracle.dijkstra(row, col, w, s)
         with sssp.Graph(row, col, w) as G:
             G.reorder()
+            G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, -1)  # heavy hubs through the chunk list too
             for d in (10, 60):
                 assert_same(G.sssp(s, d), exp, f"hub src={s} delta={d}")
                 assert G.stats()["hub_chunks"] > 0
@@ -223,6 +224,52 @@ def test_pro_matches_oracle(sssp, wt):
     assert np.array_equal(ex["rowlist"], oracle.pro_rowlist(ref["row"], ref["val"], delta))
 
 
+# --------------------------------------------- edge-balanced phase 2 -----
+@pytest.mark.parametrize("eb", [0, -1, 64])
+@pytest.mark.parametrize("wt,deltas", [("u32", (1, 8, 32, 200)), ("f32", (0.01, 0.1, 0.5))])
+@pytest.mark.parametrize("flags", [3, 0])
+def test_p2_edge_balanced_parity(sssp, eb, wt, deltas, flags):
+    """Phases 2&3 with equal heavy arcs per warp for every bucket
+    (eb=0), never (-1), or buckets of >= 64 settled entries; with and without
+    PRO (without: the whole adjacency with a per-arc heavy predicate)."""
+    g = gen.kronecker(13, 16, seed=77, weights=wt)
+    srcs = gen.sample_sources(g, 2, seed=13)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if flags:
+            G.reorder(flags)
+        G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, eb)
+        for s in srcs:
+            exp = oracle.dijkstra(g.row, g.col, g.w, int(s))
+            for d in deltas:
+                assert_same(G.sssp(int(s), d), exp, f"eb={eb} {wt} flags={flags} delta={d} src={s}")
+
+
+def test_p2_edge_balanced_hubs_and_grid(sssp):
+    """Hubs far above 4096 heavy arcs (one entry spread over many warps) and a
+    grid with hundreds of small buckets, every bucket edge-balanced."""
+    n = 30000
+    rng = np.random.default_rng(5)
+    arcs = []
+    for i in range(1, n + 1):
+        w = int(rng.integers(1, 100))
+        arcs += [(0, i, w), (i, 0, w), (1, i, w + 1), (i, 1, w + 1)]
+    row, col, w = csr_from_arcs(n + 1, arcs)
+    exp = oracle.dijkstra(row, col, w, 5)
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, 0)
+        for d in (2, 10, 50):
+            assert_same(G.sssp(5, d), exp, f"hubs delta={d}")
+    g = gen.grid(300, 200, p=0.2, seed=5)
+    s = int(gen.sample_sources(g, 1, seed=1)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, 0)
+        for d in (50, 400):
+            assert_same(G.sssp(s, d), exp, f"grid eb delta={d}")
+
+
 # ------------------------------------------------------------- stats ------
 def test_stats_invariants(sssp):
     g = gen.kronecker(13, 16, seed=8)
@@ -233,10 +280,16 @@ def test_stats_invariants(sssp):
     rl = oracle.pro_rowlist(ref["row"], ref["val"], 32)
     heavy_deg = rl[2::2] - rl[1::2]  # end - heavy per new vertex
     reach_new = exp[ref["new2old"]] != INF
-    with sssp.Graph(g.row, g.col, g.w) as G:
-        G.reorder()
-        G.sssp(s, 32)
-        st = G.stats()
+    for eb in (0, -1):  # edge-balanced phase 2 in every bucket / never
+        with sssp.Graph(g.row, g.col, g.w) as G:
+            G.reorder()
+            G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, eb)
+            G.sssp(s, 32)
+            st = G.stats()
+        _check_stats(st, reach, heavy_deg, reach_new)
+
+
+def _check_stats(st, reach, heavy_deg, reach_new):
     assert st["reachable"] == reach
     # valid updates = reachable - 1; every update is >= valid
     assert st["updates"] >= reach - 1

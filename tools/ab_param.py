@@ -16,4 +16,4 @@ with sssp.Graph(g.row, g.col, g.w) as G:
             for s in srcs: G.run(int(s), delta)
             t, n = G.kernel_time(reset=True)
             st = G.stats()
-            print(f"{cfg} param{param}={v:7d}: {t/n:.3f} ms  filtered={st['filtered_arcs']/1e6:.1f}M cover={st['bitmap_vertices']}", flush=True)
+            print(f"{cfg} param{param}={v:7d}: {t/n:.3f} ms  buckets={st['buckets']} heavy={st['heavy_arcs']/1e6:.1f}M", flush=True)
