@@ -163,10 +163,18 @@ typedef enum {
     SSSP_PARAM_SYNC = 6,           /* ablation: 1 level-synchronous phase 1 (a grid barrier per
                                       frontier level, the paper's BL); 0 the
                                       bucket-aware asynchronous phase 1 (BASYN) [0] */
-    SSSP_PARAM_P2_EDGE_BALANCED = 7 /* phases 2&3 with equal heavy arcs per warp
+    SSSP_PARAM_P2_EDGE_BALANCED = 7, /* phases 2&3 with equal heavy arcs per warp
                                       for buckets with >= value settled entries; smaller
                                       buckets (and -1 = never) relax heavy arcs through the
                                       phase-1 vertex bins [-1] */
+    SSSP_PARAM_ADAPTIVE_DELTA = 8  /* NEXT-1, Eq. (1)-(2) P:1006-1028 (Alg. 2 l.11): 0 fixed
+                                      Delta; 1 Delta_i = Delta_{i-1} + eps_i (Eq. (2) as
+                                      printed); 2 Delta_i = Delta_0 + eps_i (Fig. 6 text,
+                                      P:1033-1037). eps_i from the converged-vertex and thread
+                                      counts of the previous two buckets (reading R7: |.| bars),
+                                      Delta_i clamped to [Delta_0/4, 4 Delta_0]. The delta of
+                                      sssp_run is Delta_0. Distances do not change (Delta-
+                                      stepping is exact for every Delta) [0] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 
@@ -179,7 +187,13 @@ sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_t* launches
 /* Scheduler timeline of the last run: one entry per grid barrier (written by
  * the last CTA to arrive, before it releases the others) plus a kernel-start
  * entry (which = 99). which: 0 end of phase 1, 1 end of phases 2&3, 2/3
- * rescan stages, 4/5 sweep fall-back stages. Up to 4096 entries. */
+ * rescan stages, 4/5 sweep fall-back stages, 6 edge-balanced phase-2
+ * compaction, 7 adaptive-Delta slot merge; pad = end of the current bucket in
+ * ring-slot units (cur + 1 with a fixed Delta). With SSSP_PARAM_ADAPTIVE_DELTA
+ * every closed bucket i also adds which = 8: cur = C_i (settled vertices),
+ * tail = T_i (phase-1 queue items), mode = width of the next bucket in slots,
+ * far_min = Delta_{i+1} as binary32 bits (in slot units), pad = i + 1.
+ * Up to 4096 entries. */
 typedef struct sssp_trace_entry {
     uint64_t t_ns;   /* %globaltimer */
     uint32_t which;  /* barrier kind (see above) */

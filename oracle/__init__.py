@@ -167,3 +167,31 @@ def bucket_histogram(dist, delta, nb=4096):
     counts = np.zeros(nb, dtype=np.int64)
     n = _load().oracle_bucket_histogram(len(db), db.ctypes.data, wtype, float(delta), counts.ctypes.data, nb)
     return counts[: min(n, nb)]
+
+
+def adaptive_delta(C, T, delta0, reading="A", lo=0.25, hi=4.0):
+    """Bucket widths of the adaptive Delta variant (NEXT-1), PAPER Eq. (1)-(2)
+     step by step, reading R7 for the garbled bars:
+
+        eps_i = 0                                                   i = 0, 1
+        eps_i = |C_{i-2} - C_{i-1}| / (C_{i-2} + C_{i-1})
+                * (T_{i-2} - T_{i-1}) / (T_{i-2} + T_{i-1}) * Delta_0   i >= 2   (1)
+        Delta_i = Delta_{i-1} + eps_i                                        (2)
+
+    C_i / T_i: converged vertices / threads of bucket i. Reading
+    "B" takes the Fig. 6 text instead (bucket k ends at 25(k+1) + sum eps,
+    P:1033-1037, i.e. Delta_i = Delta_0 + eps_i). Delta_i is clamped to
+    [lo, hi] * Delta_0 (our reading; the paper states no bound). A zero
+    denominator gives eps_i = 0. Returns [Delta_0, ..., Delta_n] for the
+    n = len(C) closed buckets (Delta_i is known once bucket i-1 closes)."""
+    assert len(C) == len(T)
+    deltas = [float(delta0)]
+    for i in range(1, len(C) + 1):
+        eps = 0.0
+        if i >= 2:
+            c2, c1, t2, t1 = float(C[i - 2]), float(C[i - 1]), float(T[i - 2]), float(T[i - 1])
+            if c2 + c1 > 0 and t2 + t1 > 0:
+                eps = abs(c2 - c1) / (c2 + c1) * ((t2 - t1) / (t2 + t1)) * delta0
+        prev = deltas[-1] if reading == "A" else float(delta0)
+        deltas.append(min(max(prev + eps, lo * delta0), hi * delta0))
+    return deltas

@@ -45,6 +45,7 @@ SSSP_PARAM_L2_PERSIST = 4
 SSSP_PARAM_ADWL = 5
 SSSP_PARAM_SYNC = 6
 SSSP_PARAM_P2_EDGE_BALANCED = 7
+SSSP_PARAM_ADAPTIVE_DELTA = 8
 
 INF_U32 = 0xFFFFFFFF
 
@@ -233,7 +234,7 @@ def sssp_get_trace(h, max_entries=4096):
     for i in range(min(n.value, max_entries)):
         e = buf[i]
         out.append(dict(t_us=(e.t_ns - t0) / 1e3, which=e.which, cur=e.cur, tail=e.tail, mode=e.mode,
-                        far_min=e.far_min))
+                        far_min=e.far_min, pad=e.pad))
     return out
 
 

@@ -84,10 +84,12 @@ enum : u32 {
   MODE_SWEEP_LIGHT = 5,
   MODE_SWEEP_HEAVY = 6,
   MODE_P2_COMPACT = 7,  // edge-balanced phase 2, step 1: settled entries -> heavy-arc offsets
-  MODE_P2_RELAX = 8     // ... step 2: equal heavy-arc ranges per warp
+  MODE_P2_RELAX = 8,    // ... step 2: equal heavy-arc ranges per warp
+  MODE_MERGE = 9        // adaptive Delta: fold the slots (cur, cur_end) into slot cur
 };
 enum : u32 { ERR_OVERFLOW = 1, ERR_INTERNAL = 2 };
-enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5, SYNC_P2C = 6 };
+enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5, SYNC_P2C = 6,
+              SYNC_MG = 7, TRACE_ADAPT = 8 };
 enum : u32 { SRC_QUEUE = 0, SRC_STATIC = 1, SRC_HUB = 2, SRC_SWEEP = 3 };
 
 enum {
@@ -130,7 +132,20 @@ struct __align__(128) Ctl {
   u32 p2_begin, p2_end, err, epochs;
   u32 rescans, rescan_base, changed, sweep_first;
   u32 sweeps, trace_n, round_end, rounds;  // round_end: level-synchronous mode (ablation)
-  u32 pad_a[16];
+  // Bucket = fine ring slots [cur, cur_end) (units of the fine width g = delta_u / 1/inv_delta).
+  // Fixed Delta: cur_end = cur + 1. Adaptive Delta (NEXT-1, Eq. (1)-(2) P:1006-1028): the
+  // width m (fine slots) follows Delta_i = Delta_{i-1} + eps_i, see adapt_next().
+  u32 cur_end;
+  u32 a_mode;        // 0 fixed, 1 Eq. (2) cumulative (reading A), 2 Delta0 + eps_i (reading B)
+  u32 a_i;           // buckets completed
+  u32 a_c1, a_c2;    // C_{i-1}, C_{i-2}: converged (settled) vertices of the previous buckets
+  u32 a_t1, a_t2;    // T_{i-1}, T_{i-2}: threads (phase-1 queue items) of the previous buckets
+  float a_dlt;       // Delta_{i-1} in fine units
+  float a_d0;        // Delta_0 in fine units
+  u32 a_mmin, a_mmax, a_m;  // width clamp and current width (fine slots)
+  u32 lvl;           // light/heavy level of the current bucket: light iff w < g << lvl
+  u32 csum;          // settled vertices of the current bucket (phase 2 counts them)
+  u32 pad_a[2];
   u32 bar_count, pad3[31];   // own line: arrivals
   u32 bar_gen, pad4[31];     // own line: spun on
   u32 p2_head, pad5[31];     // own line: phase-2 static tickets
@@ -175,7 +190,8 @@ struct Params {
   u32 claim_max;
   // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
   // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL;
-  // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries).
+  // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries;
+  // bits 3/4 adaptive Delta reading A/B (NEXT-1); bit 5 f32 weights (theta level bits)).
   // Params stays <= 128 bytes: larger, it spills around the out-of-line pb_flush call.
   u32 flags;
 };
@@ -216,6 +232,7 @@ struct Smem {
   u32 claim_h, claim_n, claim_src;
   // control snapshot
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
+  u32 cur_end, rowc_off, theta_bits;  // bucket end (fine slots), light/heavy level
 };
 
 // ---------------------------------------------------------------- helpers --
@@ -335,7 +352,9 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
     const u64 e = ok ? sm.pb[w][i] : 0ULL;
     const u32 v = (u32)e, nd = (u32)(e >> 32);
     const u32 x = ok ? bucket_of_f<F32>(p, nd) : 0u;
-    if (ok && x == nearb) {
+    const u32 c0 = sm.cur;
+    const bool in_cur = x - c0 < sm.cur_end - c0;  // current bucket [cur, cur_end): its queue is slot cur
+    if (ok && nearb != NONE && in_cur) {
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
       ok = false;
@@ -346,7 +365,7 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
     }
     const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
     if (ok) {
-      const u32 s = x & p.kmask;
+      const u32 s = (in_cur ? c0 : x) & p.kmask;
       const u32 peers = __match_any_sync(m, s);
       const u32 leader = __ffs(peers) - 1;
       const u32 cnt = __popc(peers);
@@ -432,7 +451,7 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     bool take = valid[k];
-    if (!PRO) take = take && ((PH == 1) ? (a[k].y < p.delta_bits) : (a[k].y >= p.delta_bits));
+    if (!PRO) take = take && ((PH == 1) ? (a[k].y < sm.theta_bits) : (a[k].y >= sm.theta_bits));
     if (F32) {
       nd[k] = __float_as_uint(__fadd_rn(__uint_as_float(d[k]), __uint_as_float(a[k].y)));  // Alg. 1 l.1
     } else {
@@ -492,14 +511,15 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
 
 // Range of an item for phase PH: PRO -> light [start, heavy) / heavy [heavy, end);
 // no PRO -> the whole adjacency (predicate per arc).
-template <bool PRO, int PH>
-__device__ __forceinline__ void item_range(const Params& p, u32 v, i64& b, i64& e) {
-  const uint2 r = p.rowc[v];
+template <bool PRO, int PH, bool EXT>
+__device__ __forceinline__ void item_range(const Params& p, const Smem& sm, u32 v, i64& b, i64& e) {
+  const uint2* rowc = EXT ? p.rowc + sm.rowc_off : p.rowc;  // heavy offsets of the bucket's level
+  const uint2 r = rowc[v];
   if (PRO && PH == 1) {
     b = r.x;
     e = r.y;
   } else {
-    e = p.rowc[v + 1].x;
+    e = rowc[v + 1].x;
     b = (PRO && PH == 2) ? r.y : r.x;
   }
 }
@@ -515,7 +535,7 @@ __device__ __forceinline__ u32 batch_item_index(u32 r) {
 // src: SRC_QUEUE phase-1 queue, SRC_STATIC phase-2 static range, SRC_HUB
 // phase-2 hub queue, SRC_SWEEP fall-back sweep over dist[] (no queue pushes
 // into the current bucket, hubs stay in the range list).
-template <bool F32, bool PRO, int PH, int N, bool ADWL = true>
+template <bool F32, bool PRO, int PH, int N, bool ADWL = true, bool EXT = false>
 __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u64 (&it)[N],
                                               const bool (&has)[N], u32 lim, u32 src, u32 slot) {
   const u32 tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
@@ -545,7 +565,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       // Chunk items in the phase-2 static range are phase-1 work already done.
       if (!(PH == 2 && src == SRC_STATIC)) {
         i64 rb, re;
-        item_range<PRO, PH>(p, v, rb, re);
+        item_range<PRO, PH, EXT>(p, sm, v, rb, re);
         const i64 b = rb + (i64)hi * HUB_CHUNK;
         beg[i] = (u32)b;
         len[i] = (u32)min((i64)HUB_CHUNK, re - b);
@@ -561,7 +581,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       } else {
         c_settled += 1;
         i64 rb, re;
-        item_range<PRO, PH>(p, v, rb, re);
+        item_range<PRO, PH, EXT>(p, sm, v, rb, re);
         const i64 l = re - rb;
         if (!ADWL) {  // ablation: the vertex's own thread walks all its arcs
           beg[i] = (u32)rb;
@@ -633,6 +653,10 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   }
   // ---- stats (warp-aggregated)
   st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
+  if (EXT && PH == 2 && !sweep && (p.flags & 24u)) {  // adaptive Delta: C_i (converged vertices)
+    const u32 cs = __reduce_add_sync(SSSP_FULL_MASK, c_settled);
+    if (lane == 0 && cs) atomicAdd(&p.ctl->csum, cs);
+  }
   if (PH == 1) st_add(sm, ST_STALE, c_stale);
   st_add(sm, PH == 1 ? ST_LIGHT : ST_HEAVY, c_arcs);
   st_add(sm, ST_CHUNKS, c_chunks);
@@ -807,6 +831,58 @@ __device__ __forceinline__ void enter_sweep(volatile Ctl* c) {
   c->mode = MODE_SWEEP_LIGHT;
 }
 
+// Adaptive Delta (NEXT-1): PAPER Eq. (1)-(2), Alg. 2 l.11
+// Update_Delta_Epsilon, with reading R7: the garbled bars are
+// absolute values,
+//   eps_i = |C_{i-2} - C_{i-1}| / (C_{i-2} + C_{i-1})
+//           * (T_{i-2} - T_{i-1}) / (T_{i-2} + T_{i-1}) * Delta_0     (i >= 2; else 0)
+//   Delta_i = Delta_{i-1} + eps_i   (reading A; reading B: Delta_0 + eps_i, Fig. 6 text)
+// clamped to [Delta_0/4, 4 Delta_0]; C = vertices settled in the bucket
+// ("converged vertices"), T = phase-1 queue items of the bucket (one
+// thread per active vertex in the paper's master kernel). So more work
+// per bucket (T up) narrows the next bucket. Runs on the one
+// thread that closes a bucket; the next bucket spans round(Delta_i / g) fine
+// slots and its light level is the smallest g * 2^l >= that width.
+__device__ void adapt_next(const Params& p, u32 t_i) {
+  volatile Ctl* c = p.ctl;
+  const u32 c_i = c->csum;
+  c->csum = 0;
+  const u32 i = c->a_i + 1;
+  c->a_c2 = c->a_c1;
+  c->a_c1 = c_i;
+  c->a_t2 = c->a_t1;
+  c->a_t1 = t_i;
+  c->a_i = i;
+  const float d0 = c->a_d0;
+  float eps = 0.f;
+  if (i >= 2) {
+    const float c2 = (float)c->a_c2, c1 = (float)c->a_c1, t2 = (float)c->a_t2, t1 = (float)c->a_t1;
+    if (c2 + c1 > 0.f && t2 + t1 > 0.f) eps = fabsf(c2 - c1) / (c2 + c1) * ((t2 - t1) / (t2 + t1)) * d0;
+  }
+  float dl = (c->a_mode == 2 ? d0 : c->a_dlt) + eps;
+  dl = fminf(fmaxf(dl, 0.25f * d0), 4.f * d0);
+  c->a_dlt = dl;
+  u32 m = (u32)rintf(dl);
+  m = min(max(m, c->a_mmin), c->a_mmax);
+  c->a_m = m;
+  u32 l = 0;
+  while ((1u << l) < m) ++l;
+  c->lvl = l;
+  const u32 tn = c->trace_n;
+  if (tn < TRACE_CAP) {  // (C_i, T_i, next width, Delta_i) for sssp_get_trace
+    TraceEnt e;
+    e.t_ns = globaltimer();
+    e.which = TRACE_ADAPT;
+    e.cur = c_i;
+    e.tail = t_i;
+    e.mode = m;
+    e.far_min = __float_as_uint(dl);
+    e.pad = i;
+    p.trace[tn] = e;
+    c->trace_n = tn + 1;
+  }
+}
+
 // Last CTA to arrive runs the serial scheduler step (fused phase 3).
 __device__ void decide(const Params& p, u32 which) {
   volatile Ctl* c = p.ctl;
@@ -821,7 +897,7 @@ __device__ void decide(const Params& p, u32 which) {
   }
   if (which == SYNC_P1) {
     const u32 cur = c->cur, s = cur & p.kmask;
-    if (c->far_min <= cur) {  // phase-1 work was dropped (queue full)
+    if (c->far_min < c->cur_end) {  // phase-1 work was dropped (queue full)
       enter_sweep(c);
       return;
     }
@@ -850,8 +926,9 @@ __device__ void decide(const Params& p, u32 which) {
     const u32 cur = c->cur, s = cur & p.kmask;
     sc[s].p2 = c->p2_end;
     const u32 fm = c->far_min;
-    if ((u32)sc[s].word != 0) {  // f32: a heavy relaxation rounded into bucket cur
-      if (fm <= cur) {
+    if ((u32)sc[s].word != 0) {  // a heavy relaxation landed in bucket cur (f32 rounding, or
+                                 // adaptive Delta with a light level below the width)
+      if (fm < c->cur_end) {
         enter_sweep(c);
       } else {
         c->round_end = min((u32)(sc[s].word >> 32), p.cap);
@@ -861,7 +938,7 @@ __device__ void decide(const Params& p, u32 which) {
       return;
     }
     u32 nxt = NONE;
-    for (u32 x = cur + 1; x <= c->lim && x != NONE; ++x)
+    for (u32 x = c->cur_end; x <= c->lim && x != NONE; ++x)
       if ((u32)(sc[x & p.kmask].word >> 32) != 0) {
         nxt = x;
         break;
@@ -875,15 +952,23 @@ __device__ void decide(const Params& p, u32 which) {
       c->mode = MODE_RESCAN_CLEAR;
       return;
     }
+    const u32 t_items = min((u32)(sc[s].word >> 32), p.cap);  // T_i: items of bucket cur
     sc[s].word = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
     sc[s].head = 0;
     sc[s].p2 = 0;
     const u64 lim = (u64)cur + K - 1;  // excludes slot s of bucket cur+K: reset just now
     c->lim = (u32)min(lim, (u64)NONE - 1);
     c->cur = nxt;
+    if (c->a_mode) adapt_next(p, t_items);
+    c->cur_end = (u32)min((u64)nxt + c->a_m, (u64)c->lim + 1);
+    c->epochs = c->epochs + 1;
+    for (u32 x = nxt + 1; x < c->cur_end; ++x)
+      if ((u32)(sc[x & p.kmask].word >> 32) != 0) {  // entries binned before the width grew
+        c->mode = MODE_MERGE;
+        return;
+      }
     c->round_end = min((u32)(sc[nxt & p.kmask].word >> 32), p.cap);
     c->mode = MODE_PHASE1;
-    c->epochs = c->epochs + 1;
   } else if (which == SYNC_RC) {
     for (u32 s = 0; s < K; ++s) {
       sc[s].word = 0;
@@ -894,7 +979,20 @@ __device__ void decide(const Params& p, u32 which) {
     c->far_min = NONE;
     c->cur = r;
     c->lim = (u32)min((u64)r + K - 1, (u64)NONE - 1);
+    c->cur_end = (u32)min((u64)r + c->a_m, (u64)c->lim + 1);
     c->mode = MODE_RESCAN_FILL;
+  } else if (which == SYNC_MG) {  // slots (cur, cur_end) folded into slot cur
+    for (u32 x = c->cur + 1; x < c->cur_end; ++x) {
+      sc[x & p.kmask].word = 0;
+      sc[x & p.kmask].head = 0;
+      sc[x & p.kmask].p2 = 0;
+    }
+    if (c->far_min < c->cur_end) {  // slot cur overflowed while merging
+      enter_sweep(c);
+      return;
+    }
+    c->round_end = min((u32)(sc[c->cur & p.kmask].word >> 32), p.cap);
+    c->mode = MODE_PHASE1;
   } else if (which == SYNC_RF) {
     c->round_end = min((u32)(sc[c->cur & p.kmask].word >> 32), p.cap);
     c->mode = MODE_PHASE1;
@@ -908,10 +1006,18 @@ __device__ void decide(const Params& p, u32 which) {
     } else if (which == SYNC_SL) {
       c->mode = MODE_SWEEP_HEAVY;
     } else {  // bucket cur is final; rebuild the ring from dist[] for what follows
-      c->rescan_base = c->cur + 1;
+      c->rescan_base = c->cur_end;
       c->mode = MODE_RESCAN_CLEAR;
     }
   }
+}
+
+// Bucket extent and light/heavy level of the current bucket into shared memory.
+__device__ __forceinline__ void load_bucket(const Params& p, Smem& sm, volatile Ctl* vc) {
+  sm.cur_end = vc->cur_end;
+  const u32 l = vc->lvl;
+  sm.rowc_off = (p.flags & 64u) ? l * (p.V + 1) : 0u;  // levels built only with PRO
+  sm.theta_bits = l == 0 ? p.delta_bits : ((p.flags & 32u) ? p.delta_bits + (l << 23) : p.delta_bits << l);
 }
 
 __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
@@ -937,7 +1043,7 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
         e.tail = (u32)(((volatile SlotCtl*)p.sc)[vc->cur & p.kmask].word >> 32);
         e.mode = vc->mode;
         e.far_min = vc->far_min;
-        e.pad = 0;
+        e.pad = vc->cur_end;
         p.trace[tn] = e;
         vc->trace_n = tn + 1;
       }
@@ -959,6 +1065,7 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
     sm.p2_end = vc->p2_end;
     sm.sweep_first = vc->sweep_first;
     sm.round_end = vc->round_end;
+    load_bucket(p, sm, vc);
     sm.st[ST_P_BAR] += (unsigned long long)(clock64() - t_b);
   }
   __syncthreads();
@@ -1035,9 +1142,9 @@ __device__ void phase1(const Params& p, Smem& sm) {
       }
     }
     if (!ABL || (p.flags & 1u))
-      process_batch<F32, PRO, 1, IPT>(p, sm, it, has, lim, SRC_QUEUE, slot);
+      process_batch<F32, PRO, 1, IPT, true, ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
     else
-      process_batch<F32, PRO, 1, IPT, !ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
+      process_batch<F32, PRO, 1, IPT, !ABL, ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
     if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
   }
 }
@@ -1115,9 +1222,9 @@ __device__ void phase2(const Params& p, Smem& sm) {
       st_relaxed_u64(base_q + batch_item_index(i), SENTINEL);  // recycle the queue entry
     }
     if (!ABL || (p.flags & 1u))
-      process_batch<F32, PRO, 2, IPT2>(p, sm, it, has, lim, src, slot);
+      process_batch<F32, PRO, 2, IPT2, true, ABL>(p, sm, it, has, lim, src, slot);
     else
-      process_batch<F32, PRO, 2, IPT2, !ABL>(p, sm, it, has, lim, src, slot);
+      process_batch<F32, PRO, 2, IPT2, !ABL, ABL>(p, sm, it, has, lim, src, slot);
     if (threadIdx.x == 0) atomicAdd(&c->hub_word, (u64)0 - (u64)n);
   }
 }
@@ -1169,9 +1276,10 @@ __device__ void p2_compact(const Params& p, Smem& sm) {
       st[i] = 0;
       if (has[i] && (u32)(e[i] >> 32) == cd[i]) {  // final in this bucket
         const u32 v = (u32)e[i];
-        const uint2 r = p.rowc[v];
+        const uint2* rowc = p.rowc + sm.rowc_off;
+        const uint2 r = rowc[v];
         st[i] = PRO ? r.y : r.x;
-        hl[i] = p.rowc[v + 1].x - st[i];
+        hl[i] = rowc[v + 1].x - st[i];
         ++c_live;
         c_arcs += hl[i];
         if (hl[i]) x += (1ULL << 32) | hl[i];
@@ -1211,6 +1319,10 @@ __device__ void p2_compact(const Params& p, Smem& sm) {
   }
   st_add(sm, ST_HEAVYV, c_live);
   st_add(sm, ST_HEAVY, c_arcs);
+  if (p.flags & 24u) {
+    const u32 cs = __reduce_add_sync(SSSP_FULL_MASK, c_live);
+    if (lane == 0 && cs) atomicAdd(&p.ctl->csum, cs);
+  }
 }
 
 template <bool F32, bool PRO>
@@ -1357,7 +1469,7 @@ __device__ void rescan_fill(const Params& p, Smem& sm) {
 // style sweeps over all v with bucket(dist[v]) == cur until nothing in the
 // bucket improves (light arcs; xd[] skips vertices unchanged since their last
 // expansion), then one sweep over heavy arcs. Always makes progress.
-template <bool F32, bool PRO, int PH>
+template <bool F32, bool PRO, int PH, bool EXT>
 __device__ void sweep(const Params& p, Smem& sm) {
   const u32 cur = sm.cur, lim = sm.lim;
   const bool first = sm.sweep_first != 0;
@@ -1372,7 +1484,8 @@ __device__ void sweep(const Params& p, Smem& sm) {
       it[i] = SENTINEL;
       if (v < p.V) {
         const u32 d = ld_cg(p.dist + v);
-        if (d != inf && bucket_of<F32>(p, d) == cur) {
+        const u32 bx = d != inf ? bucket_of<F32>(p, d) : NONE;
+        if (bx >= cur && bx < sm.cur_end) {
           if (PH == 1) {
             if (first || d < ld_cg(p.xd + v)) {
               st_relaxed_u32(p.xd + v, d);
@@ -1385,12 +1498,50 @@ __device__ void sweep(const Params& p, Smem& sm) {
         }
       }
     }
-    process_batch<F32, PRO, PH, IPT>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);
+    process_batch<F32, PRO, PH, IPT, true, EXT>(p, sm, it, has, lim, SRC_SWEEP, cur & p.kmask);
   }
 }
 
-// ABL = ablation build (SSSP_PARAM_ADWL = 0 / SSSP_PARAM_SYNC = 1 paths compiled in);
-// the default kernel (ABL = false) carries none of that code.
+// Adaptive Delta: the bucket grew over slots (cur, cur_end) that already hold
+// entries pushed while they were far buckets. Move the live ones into slot cur
+// (pb_flush resolves them to the current bucket); stale ones are dropped (a
+// better entry of the same vertex was pushed when dist[] improved).
+template <bool F32>
+__device__ void merge_slots(const Params& p, Smem& sm) {
+  const u32 cur = sm.cur, ce = sm.cur_end, lim = sm.lim, lane = lane_id();
+  u32 moved = 0;
+  const i64 t0 = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL;
+  const i64 nt = (i64)gridDim.x * blockDim.x;
+  for (u32 x = cur + 1; x < ce; ++x) {
+    const u32 sl = x & p.kmask;
+    const u32 tail = min((u32)(ld_relaxed_u64(&p.sc[sl].word) >> 32), p.cap);
+    u64* q = p.items + (u64)sl * p.cap;
+    for (i64 b = t0; b < tail; b += nt) {
+      const i64 i = b + lane;
+      bool want[UNROLL] = {};
+      u32 vv[UNROLL] = {}, dd[UNROLL] = {};
+      if (i < tail) {
+        const u64 e = ld_relaxed_u64(q + i);
+        st_relaxed_u64(q + i, SENTINEL);
+        if (e != SENTINEL) {
+          vv[0] = (u32)e;
+          dd[0] = (u32)(e >> 32);
+          want[0] = ld_cg(p.dist + vv[0]) == dd[0];
+        }
+      }
+      moved += want[0];
+      stage_pushes<F32>(p, sm, lim, NONE, want, vv, dd);
+    }
+  }
+  if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
+  const u32 mv = __reduce_add_sync(SSSP_FULL_MASK, moved);
+  if (lane == 0 && mv) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)(-(long long)mv));  // not updates
+}
+
+// ABL = extended build: the ablation paths (SSSP_PARAM_ADWL = 0 / SSSP_PARAM_SYNC = 1),
+// the edge-balanced phase 2 and the adaptive-Delta slot merge are compiled in; the
+// default kernel (ABL = false) carries none of that code (it raised the default
+// kernel's register spills from 164 to 288 bytes and cost ~6 % on C4).
 template <bool F32, bool PRO, bool ABL>
 __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) {
   __shared__ Smem sm;
@@ -1410,6 +1561,7 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     sm.p2_end = vc->p2_end;
     sm.sweep_first = vc->sweep_first;
     sm.round_end = vc->round_end;
+    load_bucket(p, sm, vc);
   }
   __syncthreads();
   for (;;) {
@@ -1421,11 +1573,14 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     } else if (mode == MODE_PHASE2) {
       phase2<F32, PRO, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
-    } else if (mode == MODE_P2_COMPACT) {
-      p2_compact<F32, PRO>(p, sm);
+    } else if (ABL && mode == MODE_MERGE) {  // extended build only (adaptive Delta)
+      if constexpr (ABL) merge_slots<F32>(p, sm);
+      grid_barrier(p, sm, SYNC_MG);
+    } else if (ABL && mode == MODE_P2_COMPACT) {  // extended build only (edge-balanced phase 2)
+      if constexpr (ABL) p2_compact<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2C);
-    } else if (mode == MODE_P2_RELAX) {
-      p2_relax<F32, PRO>(p, sm);
+    } else if (ABL && mode == MODE_P2_RELAX) {
+      if constexpr (ABL) p2_relax<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (mode == MODE_RESCAN_CLEAR) {
       rescan_clear(p);
@@ -1434,10 +1589,10 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
       rescan_fill<F32>(p, sm);
       grid_barrier(p, sm, SYNC_RF);
     } else if (mode == MODE_SWEEP_LIGHT) {
-      sweep<F32, PRO, 1>(p, sm);
+      sweep<F32, PRO, 1, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_SL);
     } else {
-      sweep<F32, PRO, 2>(p, sm);
+      sweep<F32, PRO, 2, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_SH);
     }
   }
@@ -1453,7 +1608,12 @@ __global__ void k_fill_u32(u32* __restrict__ a, i64 n, u32 v) {
 }
 
 // Alg. 2 l.1-3: dist[s] = 0, bucket 0 queue holds (s, 0), counters reset.
-__global__ void k_seed(Params p, u32 src) {
+struct AdaptInit {
+  u32 mode;        // 0 fixed Delta, 1 / 2 adaptive (readings A / B of Eq. (2))
+  float d0;        // Delta_0 in fine units
+  u32 m0, mmin, mmax, lvl0;
+};
+__global__ void k_seed(Params p, u32 src, AdaptInit ai) {
   const u32 t = threadIdx.x;
   for (u32 s = t; s < p.K; s += blockDim.x) {
     p.sc[s].word = 0;
@@ -1485,6 +1645,17 @@ __global__ void k_seed(Params p, u32 src) {
     c->trace_n = 0;
     c->round_end = 1;
     c->rounds = 0;
+    c->cur_end = ai.m0;
+    c->a_mode = ai.mode;
+    c->a_i = 0;
+    c->a_c1 = c->a_c2 = c->a_t1 = c->a_t2 = 0;
+    c->a_dlt = ai.d0;
+    c->a_d0 = ai.d0;
+    c->a_mmin = ai.mmin;
+    c->a_mmax = ai.mmax;
+    c->a_m = ai.m0;
+    c->lvl = ai.lvl0;
+    c->csum = 0;
   }
 }
 

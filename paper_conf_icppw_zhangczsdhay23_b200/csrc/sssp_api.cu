@@ -41,6 +41,9 @@ struct sssp_graph_s {
   longlong2* rowp = nullptr;  // [V+1] {start, heavy}
   uint2* rowc = nullptr;      // [V+1] compact copy for the persistent kernel
   bool rowc_valid = false;
+  uint2* rowc_lv = nullptr;   // [5][V+1] adaptive Delta: heavy offsets for light levels g << l
+  bool rowc_lv_valid = false;
+  u32 rowc_lv_g = 0;          // fine-unit bits the levels were built for
   uint2* arcs = nullptr;      // [A]
   u32 maxw_bits = 0;
   u32* old2new = nullptr;  // null until PRO_DEGREE
@@ -74,7 +77,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -220,7 +223,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
   void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
-                  g->items, g->hub_items, g->p2o, g->stats, g->trace, g->out_tmp};
+                  g->items, g->hub_items, g->p2o, g->rowc_lv, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& e : g->ev)
@@ -290,6 +293,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_P2_EDGE_BALANCED:
       if (v < -1 || v > 0xFFFFFF) return fail(SSSP_ERR_INVALID_ARGUMENT, "p2 edge-balanced threshold in [-1, 2^24)");
       g->p_p2eb = v;
+      return SSSP_OK;
+    case SSSP_PARAM_ADAPTIVE_DELTA:
+      if (v < 0 || v > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "adaptive delta is 0, 1 or 2");
+      g->p_adapt = v;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
@@ -433,6 +440,7 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   g->pro_flags |= flags;
   g->heavy_valid = false;
   g->rowc_valid = false;
+  g->rowc_lv_valid = false;
   g->have_result = false;
   g->reorder_timed = true;
   return SSSP_OK;
@@ -447,9 +455,40 @@ struct DeltaParams {
   u32 delta_u, delta_bits;
   float inv;
   double ahead;  // max weight / Delta (buckets a heavy push can skip ahead)
+  AdaptInit ai;  // fixed Delta: mode 0, one ring slot per bucket
 };
 
+// Adaptive Delta (NEXT-1): ring slots become fine slots of width g = Delta_0 / 4
+// (u32: max(1, floor(Delta_0 / 4))); a bucket spans m in [Delta_0/4, 4 Delta_0] / g
+// of them (at most 16), and delta_u / inv / delta_bits describe g instead of Delta.
+static void adapt_params(sssp_graph_t g, int mode, DeltaParams* dp) {
+  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
+  if (!mode || dp->delta_bits == 0xFFFFFFFFu || (g->wtype == SSSP_WEIGHT_F32 && dp->inv == 0.f)) return;
+  double d0;
+  if (g->wtype == SSSP_WEIGHT_U32) {
+    const u32 D = dp->delta_u, gu = std::max<u32>(1u, D / 4);
+    dp->delta_u = dp->delta_bits = gu;
+    d0 = (double)D / gu;
+    dp->ahead = (double)g->maxw_bits / gu;
+  } else {
+    float df;
+    memcpy(&df, &dp->delta_bits, 4);
+    const float gf = df * 0.25f;  // exact (power-of-two scale) unless subnormal
+    if (!(gf > 0.f) || gf * 4.f != df) return;
+    memcpy(&dp->delta_bits, &gf, 4);
+    dp->inv = (float)(1.0 / (double)gf);
+    d0 = 4.0;
+    dp->ahead *= 4.0;
+  }
+  const u32 mmin = std::max<u32>(1u, (u32)std::lrint(d0 / 4)), mmax = std::min<u32>(16u, (u32)std::lrint(4 * d0));
+  const u32 m0 = std::min(std::max((u32)std::lrint(d0), mmin), mmax);
+  u32 l = 0;
+  while ((1u << l) < m0) ++l;
+  dp->ai = AdaptInit{(u32)mode, (float)d0, m0, mmin, mmax, l};
+}
+
 static sssp_status delta_params(sssp_graph_t g, double delta, DeltaParams* dp) {
+  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
   if (std::isnan(delta) || delta <= 0.0) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta must be > 0 (got %g)", delta);
   if (g->wtype == SSSP_WEIGHT_U32) {
     double c = std::ceil(delta);
@@ -533,12 +572,13 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   // ring size: enough slots for the farthest heavy push (+ the recycled slot)
   u32 K = (u32)g->p_ring;
   if (K == 0) {
-    double need = std::ceil(dp.ahead) + 3.0;
+    double need = std::ceil(dp.ahead) + dp.ai.mmax + 2.0;
     K = 8;
-    while (K < need && K < 32) K <<= 1;
+    while (K < need && K < (dp.ai.mode ? 64u : 32u)) K <<= 1;
   }
   u32 cap = (u32)g->p_cap;
-  if (cap == 0) cap = (u32)std::min<i64>(2 * g->V + g->V / 2 + 65536, 0x7FFFFFFF);  // 2.5 V: far buckets collect repeated improvements
+  if (cap == 0)  // 2.5 V: far buckets collect repeated improvements; adaptive: 4x the slots, 1.5 V each
+    cap = (u32)std::min<i64>((dp.ai.mode ? g->V + g->V / 2 : 2 * g->V + g->V / 2) + 65536, 0x7FFFFFFF);
   sssp_status st = ensure_run_buffers(g, K, cap);
   if (st) return st;
   g->K_used = K;
@@ -561,14 +601,29 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
     }
     cudaGetLastError();
   }
-  ds_kernel_t kern = pick_kernel(f32, pro, g->p_adwl == 0 || g->p_sync != 0);
+  const bool adapt = dp.ai.mode != 0;
+  if (adapt && pro && (!g->rowc_lv_valid || g->rowc_lv_g != dp.delta_bits)) {
+    // heavy offsets for the light levels g << l (u32) / g * 2^l (f32), l = 0..4
+    if (!g->rowc_lv) CU(cudaMalloc(&g->rowc_lv, sizeof(uint2) * 5 * (size_t)(g->V + 1)));
+    for (u32 l = 0; l < 5; ++l) {
+      const u32 th = f32 ? dp.delta_bits + (l << 23) : dp.delta_bits << l;
+      k_heavy_offsets<<<grid_for(g->V), 256, 0, s>>>(g->rowp, g->arcs, g->V, th);
+      k_make_rowc<<<grid_for(g->V + 1), 256, 0, s>>>(g->rowp, g->V, g->rowc_lv + (size_t)l * (g->V + 1));
+      g->heavy_bits = th;
+    }
+    CU(cudaGetLastError());
+    g->rowc_lv_valid = true;
+    g->rowc_lv_g = dp.delta_bits;
+    g->rowc_valid = false;
+  }
+  ds_kernel_t kern = pick_kernel(f32, pro, g->p_adwl == 0 || g->p_sync != 0 || adapt || g->p_p2eb >= 0);
   int per_sm = 0;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, DS_THREADS, 0));
   if (per_sm < 1) return fail(SSSP_ERR_INTERNAL, "persistent kernel cannot be resident");
   if (g->p_ctas > 0) per_sm = std::min<int>(per_sm, (int)g->p_ctas);
   g->grid_ctas = per_sm * g->num_sms;
   Params p;
-  p.rowc = g->rowc;
+  p.rowc = (adapt && pro) ? g->rowc_lv : g->rowc;
   p.arcs = g->arcs;
   p.dist = g->dist;
   p.xd = g->xd;
@@ -591,9 +646,11 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.flags = (g->p_adwl ? 1u : 0u) | (g->p_sync ? 2u : 0u);
   // edge-balanced phase 2 (not in the static thread-per-vertex ablation)
   if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
+  if (adapt) p.flags |= (dp.ai.mode == 2 ? 16u : 8u) | (pro ? 64u : 0u);
+  if (f32) p.flags |= 32u;
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
-  k_seed<<<1, 64, 0, s>>>(p, src_internal);
+  k_seed<<<1, 64, 0, s>>>(p, src_internal, dp.ai);
   CU(cudaGetLastError());
   cudaEvent_t e0, e1;
   for (int i = 0; i < 2; ++i) {
@@ -646,6 +703,7 @@ extern "C" sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta) {
   if (source < 0 || source >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source %lld out of range", (long long)source);
   DeltaParams dp;
   if ((st = delta_params(g, delta, &dp))) return st;
+  adapt_params(g, (int)g->p_adapt, &dp);
   DeviceGuard dg(g->device);
   const u32 src = g->h_old2new.empty() ? (u32)source : g->h_old2new[source];
   g->have_result = false;
@@ -706,6 +764,7 @@ extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, in
     return fail(SSSP_ERR_INVALID_ARGUMENT, "bad batch arguments");
   DeltaParams dp;
   if ((st = delta_params(g, delta, &dp))) return st;
+  adapt_params(g, (int)g->p_adapt, &dp);
   for (i64 i = 0; i < n; ++i)
     if (sources[i] < 0 || sources[i] >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source[%lld] out of range", (long long)i);
   DeviceGuard dg(g->device);

@@ -2,6 +2,8 @@
 element, on seeded inputs. u32 distances must be bit-exact; f32 distances are
 bit-exact too (the f32 result is the unique min over left-to-right binary32
 path sums), which is stricter than north_star's 1e-6."""
+import math
+
 import numpy as np
 import pytest
 
@@ -401,3 +403,55 @@ def test_ablation_modes_parity(sssp, sync, adwl, flags, wt):
                 assert st["levels"] > 0
             if not adwl:
                 assert st["hub_chunks"] == 0 and st["bin_warp"] == 0 and st["bin_cta"] == 0
+
+
+# ------------------------------------------------ adaptive Delta (NEXT-1) --
+@pytest.mark.parametrize("mode", [1, 2])
+@pytest.mark.parametrize("wt,deltas", [("u32", (1, 3, 16, 64)), ("f32", (0.05, 0.1, 0.4))])
+@pytest.mark.parametrize("flags", [3, 0])
+def test_adaptive_delta_parity(sssp, mode, wt, deltas, flags):
+    """Eq. (1)-(2) bucket widths leave the distances unchanged
+    (Delta-stepping is exact for every Delta), with PRO (light
+    levels from the heavy-offset table per level) and without (predicate)."""
+    g = gen.kronecker(13, 16, seed=91, weights=wt)
+    srcs = gen.sample_sources(g, 2, seed=17)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if flags:
+            G.reorder(flags)
+        G.set_param(sssp.SSSP_PARAM_ADAPTIVE_DELTA, mode)
+        for s in srcs:
+            exp = oracle.dijkstra(g.row, g.col, g.w, int(s))
+            for d in deltas:
+                assert_same(G.sssp(int(s), d), exp, f"adaptive={mode} {wt} flags={flags} delta={d} src={s}")
+
+
+def _adapt_records(tr):
+    return [e for e in tr if e["which"] == 8]
+
+
+@pytest.mark.parametrize("mode,reading", [(1, "A"), (2, "B")])
+def test_adaptive_delta_follows_eq1(sssp, mode, reading):
+    """The widths the kernel used are the oracle's Eq. (1)-(2) applied to the
+    kernel's own per-bucket counts C_i (settled) and T_i (phase-1 items)."""
+    g = gen.grid(400, 300, p=0.2, seed=8)  # many buckets
+    s = int(gen.sample_sources(g, 1, seed=3)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_ADAPTIVE_DELTA, mode)
+        assert_same(G.sssp(s, 400), exp, "grid adaptive")
+        recs = _adapt_records(G.trace())
+        st = G.stats()
+    assert len(recs) >= 20 and st["rescans"] == 0
+    C = [r["cur"] for r in recs]
+    T = [r["tail"] for r in recs]
+    ref = oracle.adaptive_delta(C, T, 4.0, reading)  # Delta_0 = 400 = 4 ring slots of g = 100
+    got = [float(np.array([r["far_min"]], dtype=np.uint32).view(np.float32)[0]) for r in recs]
+    for i, (a, b) in enumerate(zip(got, ref[1:])):
+        assert abs(a - b) <= 1e-4 * max(1.0, abs(b)), f"Delta_{i + 1}: kernel {a} oracle {b}"
+        m = recs[i]["mode"]
+        want = min(max(int(round(b)), 1), 16)
+        assert m == want or abs(b - math.floor(b) - 0.5) < 1e-3, f"width {i + 1}: {m} vs {want}"
+    assert len(set(r["mode"] for r in recs)) > 1, "Delta never changed"
+    # C_i counts each settled vertex once (the last bucket closes without a record)
+    assert sum(C) <= int((exp != INF).sum())
