@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--sources", type=int, default=64)
     ap.add_argument("--ctas-per-sm", type=int, default=0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/cpu/e2e)")
+    ap.add_argument("--multi", action="store_true",
+                    help="NEXT-4: a step is one group of up to 32 of the rank's sources through sssp_run_multi")
     return ap.parse_args()
 
 
@@ -242,6 +244,9 @@ def main():
         torch.cuda.synchronize(dev)
         reorder_ms = G.stats()["reorder_ms"]
     inf = 0x7F800000 if g.wtype == "f32" else 0xFFFFFFFF
+    if args.multi:
+        return bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, stream,
+                           reorder, reorder_ms, t_gen, inf)
 
     def step(k):
         G.run(int(mine[k % len(mine)]), delta)
@@ -365,6 +370,119 @@ def main():
         "clocks": sampler.summary() if not args.profile else None,
         "last_run_stats": {k: st[k] for k in ("updates", "light_arcs", "heavy_arcs", "vertices_settled",
                                               "stale_items", "hub_chunks", "buckets", "rescans", "reachable")},
+    }
+    print(json.dumps(line), flush=True)
+    G.close()
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+def multi_alg_bytes(g, dist_bits, inf, lanes):
+    """Algorithmic bytes of one sssp_run_multi group (NEXT-4 design):
+    every reachable vertex expanded once -> its arcs streamed once (8 B) and one
+    128-byte D row probed per arc; one row read per expansion + 16 B of queue
+    traffic; init of D and Q (132 B per vertex) and the output gather (128 B row
+    read + 4 B per source per vertex)."""
+    reach = dist_bits != inf
+    deg = np.diff(g.row)
+    A_r, V_r = int(deg[reach].sum()), int(reach.sum())
+    return 136 * A_r + 144 * V_r + (132 + 128 + 4 * lanes) * g.V, A_r, V_r
+
+
+def bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, stream, reorder, reorder_ms,
+                t_gen, inf):
+    """NEXT-4 bench: each step runs one group of <= 32 of this rank's sources
+    through sssp_run_multi (one persistent launch); value = sources*m / time."""
+    import torch
+
+    L = 32
+    groups = [list(mine[i:i + L]) for i in range(0, len(mine), L)] or [[]]
+    out = torch.empty((L, g.V), dtype=torch.int32, device=f"cuda:{dev}")
+
+    def step(k):
+        G.run_multi(groups[k % len(groups)], delta, out)
+
+    for k in range(args.warmup):
+        step(k)
+    torch.cuda.synchronize(dev)
+    G.kernel_time(reset=True)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize(dev)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(dev)
+    with sampler if not args.profile else _Null():
+        ev0.record(stream)
+        for k in range(args.steps):
+            step(args.warmup + k)
+        ev1.record(stream)
+        ev1.synchronize()
+    torch.cuda.synchronize(dev)
+    t_ms = ev0.elapsed_time(ev1)
+    kt_total, kt_n = G.kernel_time(reset=True)
+    n_src = sum(len(groups[(args.warmup + k) % len(groups)]) for k in range(args.steps))
+    tot = torch.tensor([t_ms, float(n_src)], device=tdev)
+    if world > 1:
+        t_max = tot[:1].clone()
+        torch.distributed.all_reduce(t_max, op=torch.distributed.ReduceOp.MAX)
+        torch.distributed.all_reduce(tot, op=torch.distributed.ReduceOp.SUM)
+        t_ms, n_all = float(t_max.item()), float(tot[1].item())
+    else:
+        n_all = float(n_src)
+    value = n_all * g.m / (t_ms * 1e-3) / 1e9
+    ms = G.multi_stats()
+    e2e = None
+    if not args.no_e2e and not args.profile and world == 1:
+        grp = groups[0]
+        pinned = torch.empty((len(grp), g.V), dtype=torch.int32).pin_memory()
+        G.run_multi(grp, delta, out)
+        pinned.copy_(out[:len(grp)])
+        ne = min(args.steps, 4)
+        t0 = time.perf_counter()
+        for k in range(ne):
+            G.run_multi(grp, delta, out)  # sources host -> device inside the call
+            pinned.copy_(out[:len(grp)])  # D2H of the distance rows (synchronises)
+        te = time.perf_counter() - t0
+        e2e = {"value": round(ne * len(grp) * g.m / te / 1e9, 4), "unit": "GTEPS",
+               "h2d_bytes_per_step": 8 * len(grp), "d2h_bytes_per_step": 4 * g.V * len(grp),
+               "note": "graph resident; per step: source ids in, the group's distance rows out to pinned "
+                       "host memory; wall clock"}
+    if rank != 0:
+        if world > 1:
+            torch.distributed.barrier()
+            torch.distributed.destroy_process_group()
+        return
+    row0 = out[0].cpu().numpy().view(np.uint32)
+    b_alg, A_r, V_r = multi_alg_bytes(g, row0, inf, len(groups[0]))
+    kt_avg = kt_total / max(kt_n, 1)
+    peak, peak_kind = measured_peak()
+    achieved = b_alg / (kt_avg * 1e-3) / 1e9
+    cpu = None
+    if not args.no_cpu_baseline and not args.profile and world == 1:
+        cpu = cpu_baseline(g, sources)
+    line = {
+        "metric": METRIC, "value": round(value, 4), "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(t_ms / args.steps, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32" if g.wtype == "u32" else "f32",
+        "data": "synthetic",
+        "config": {"workload": desc + f"; multi-source batch ({len(sources)} sources, <= 32 per persistent "
+                                      "launch, sssp_run_multi, NEXT-4)",
+                   "V": g.V, "m_edges": g.m, "arcs": g.A, "delta": delta, "reorder": reorder,
+                   "reorder_ms": reorder_ms, "sources": len(sources), "sources_per_step": len(groups[0]),
+                   "parallelism": f"replicas x{world} (sources sharded, graph replicated)",
+                   "l2": "inputs larger than L2 (D rows %.2f GB, arcs %.2f GB > 126 MB L2); D re-initialised "
+                         "every step" % (128 * g.V / 1e9, 8 * g.A / 1e9), "gen_s": round(t_gen, 1)},
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": None, "peak_kind": peak_kind,
+                     "kernel": "k_ms_step (persistent, 32 sources)", "kernel_ms_avg": round(kt_avg, 4),
+                     "kernel_share_of_step": round(kt_total / t_ms, 4), "alg_bytes_per_launch": int(b_alg)},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": 4 * args.steps,
+        "clocks": sampler.summary() if not args.profile else None,
+        "last_group_stats": ms,
     }
     print(json.dumps(line), flush=True)
     G.close()

@@ -116,6 +116,24 @@ sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream);
 sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                            void* out_dev, int64_t ld);
 
+/* NEXT-4 (beyond the paper): the same batch as sssp_run_batch
+ * (row i = distances from sources[i], original ids, out_dev + i*ld, ld >= V,
+ * device buffer) computed 32 sources per persistent launch: distances are
+ * kept as D[v][32] (128-byte rows), so one arc read and one coalesced row
+ * probe serve 32 sources. Work items are vertices queued in Delta-width
+ * buckets by their smallest improved distance; an expansion relaxes every
+ * finite lane (label-correcting: exact, identical to sssp_run per source for
+ * u32 and f32). Allocates 132 B per vertex plus the ring on first use.
+ * Synchronises once per group of 32 sources. Errors as sssp_run. */
+sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
+                           void* out_dev, int64_t ld);
+
+/* Counters of the last sssp_run_multi group: out[0] successful lane updates,
+ * [1] arcs relaxed (each for all 32 lanes), [2] vertex expansions, [3] stale
+ * queue items, [4] split items (256-arc pieces), [5] buckets, [6] rescans.
+ * Writes min(n, 7) values. SSSP_ERR_INVALID_STATE before the first call. */
+sssp_status sssp_multi_stats(sssp_graph_t g, uint64_t* out, int64_t n);
+
 /* Counters of the last run (the work-efficiency metric of P:410-413 and
  * updates = successful atomicMin writes; a valid update is one
  * that writes the final distance, so valid = reachable - 1). Synchronises. */

@@ -54,7 +54,7 @@ EXPORTS = (
     "sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
-    "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile",
+    "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile", "sssp_run_multi", "sssp_multi_stats",
 )
 
 
@@ -83,6 +83,8 @@ _lib.sssp_last_error.argtypes = []
 _lib.sssp_last_error.restype = ctypes.c_char_p
 _lib.sssp_set_stream.argtypes = [_P, _P]
 _lib.sssp_run_batch.argtypes = [_P, _P, _I64, _D, _P, _I64]
+_lib.sssp_run_multi.argtypes = [_P, _P, _I64, _D, _P, _I64]
+_lib.sssp_multi_stats.argtypes = [_P, _P, _I64]
 _lib.sssp_get_stats.argtypes = [_P, ctypes.POINTER(sssp_stats)]
 _lib.sssp_export_csr.argtypes = [_P, _D, _P, _P, _P, _P]
 _lib.sssp_set_param.argtypes = [_P, _I, _I64]
@@ -102,7 +104,8 @@ _lib.sssp_get_trace.restype = _I
 _lib.sssp_get_profile.argtypes = [_P, _P, _I]
 _lib.sssp_get_profile.restype = _I
 for _n in ("sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
-           "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param"):
+           "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param",
+           "sssp_run_multi", "sssp_multi_stats"):
     getattr(_lib, _n).restype = _I
 
 
@@ -194,6 +197,21 @@ def sssp_run_batch(h, sources, delta, out_dev, ld):
     if kind != SSSP_MEM_DEVICE:
         raise ValueError("batch output must be a CUDA tensor")
     _check(_lib.sssp_run_batch(h, src.ctypes.data, len(src), float(delta), p, int(ld)), "sssp_run_batch")
+
+
+def sssp_run_multi(h, sources, delta, out_dev, ld):
+    src = np.ascontiguousarray(sources, dtype=np.int64)
+    p, kind = _ptr(out_dev)
+    if kind != SSSP_MEM_DEVICE:
+        raise ValueError("batch output must be a CUDA tensor")
+    _check(_lib.sssp_run_multi(h, src.ctypes.data, len(src), float(delta), p, int(ld)), "sssp_run_multi")
+
+
+def sssp_multi_stats(h):
+    out = np.zeros(7, dtype=np.uint64)
+    _check(_lib.sssp_multi_stats(h, out.ctypes.data, 7), "sssp_multi_stats")
+    return dict(zip(("updates", "arcs", "expansions", "stale", "split_items", "buckets", "rescans"),
+                    (int(x) for x in out)))
 
 
 def sssp_get_stats(h):
@@ -297,6 +315,13 @@ class Graph:
 
     def run_batch(self, sources, delta, out_dev, ld=None):
         sssp_run_batch(self.h, sources, delta, out_dev, ld or self.V)
+
+    def run_multi(self, sources, delta, out_dev, ld=None):
+        """NEXT-4: the batch computed 32 sources per persistent launch."""
+        sssp_run_multi(self.h, sources, delta, out_dev, ld or self.V)
+
+    def multi_stats(self):
+        return sssp_multi_stats(self.h)
 
     def stats(self):
         return sssp_get_stats(self.h)

@@ -14,6 +14,7 @@
 
 #include "../../include/sssp.h"
 #include "delta_step.cuh"
+#include "multi_source.cuh"
 #include "pro.cuh"
 #include "sort.cuh"
 
@@ -60,6 +61,15 @@ struct sssp_graph_s {
   u64* items = nullptr;
   u64* hub_items = nullptr;
   u32* p2o = nullptr;  // [cap] + uint2 [cap]: edge-balanced phase-2 scratch
+  // batched multi-source kernel (NEXT-4, sssp_run_multi)
+  u32* ms_D = nullptr;     // [V][32]
+  u32* ms_Q = nullptr;     // [V]
+  u64* ms_items = nullptr; // [ms_K * ms_cap]
+  SlotCtl* ms_sc = nullptr;
+  MCtl* ms_ctl = nullptr;
+  unsigned long long* ms_stats = nullptr;
+  u32* ms_src = nullptr;   // [32]
+  u32 ms_K = 0, ms_cap = 0;
   u32* out_tmp = nullptr;  // [V] staging for sssp_distances into pageable host memory
   unsigned long long* stats = nullptr;
   TraceEnt* trace = nullptr;
@@ -223,7 +233,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
   void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
-                  g->items, g->hub_items, g->p2o, g->rowc_lv, g->stats, g->trace, g->out_tmp};
+                  g->items, g->hub_items, g->p2o, g->rowc_lv, g->ms_D, g->ms_Q, g->ms_items, g->ms_sc, g->ms_ctl, g->ms_stats, g->ms_src, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& e : g->ev)
@@ -777,6 +787,124 @@ extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, in
     k_output<<<grid_for(g->V), 256, 0, g->stream>>>(g->dist, g->old2new, g->V, (u32*)out_dev + (size_t)i * ld);
     CU(cudaGetLastError());
   }
+  return SSSP_OK;
+}
+
+// NEXT-4: up to 32 sources per persistent launch (multi_source.cuh).
+extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
+                                      void* out_dev, int64_t ld) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (n < 0 || (n > 0 && (!sources || !out_dev)) || ld < g->V)
+    return fail(SSSP_ERR_INVALID_ARGUMENT, "bad batch arguments");
+  DeltaParams dp;
+  if ((st = delta_params(g, delta, &dp))) return st;
+  for (i64 i = 0; i < n; ++i)
+    if (sources[i] < 0 || sources[i] >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source[%lld] out of range", (long long)i);
+  if (n == 0) return SSSP_OK;
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  const bool f32 = g->wtype == SSSP_WEIGHT_F32;
+  if (!g->rowc_valid) {  // only the .x (row start) column is used here
+    k_make_rowc<<<grid_for(g->V + 1), 256, 0, s>>>(g->rowp, g->V, g->rowc);
+    CU(cudaGetLastError());
+    g->rowc_valid = true;
+  }
+  u32 K = 8;
+  while (K < std::ceil(dp.ahead) + 2.0 && K < 64) K <<= 1;
+  const u32 cap = (u32)std::min<i64>(g->V + g->V / 2 + g->A / 128 + 65536, 0x7FFFFFFF);
+  if (!g->ms_D) {
+    CU(cudaMalloc(&g->ms_D, sizeof(u32) * MS_LANES * (size_t)g->V));
+    CU(cudaMalloc(&g->ms_Q, sizeof(u32) * (size_t)g->V));
+    CU(cudaMalloc(&g->ms_ctl, sizeof(MCtl)));
+    CU(cudaMemsetAsync(g->ms_ctl, 0, sizeof(MCtl), s));
+    CU(cudaMalloc(&g->ms_stats, sizeof(unsigned long long) * MST_N));
+    CU(cudaMalloc(&g->ms_src, sizeof(u32) * MS_LANES));
+  }
+  if (K > g->ms_K || cap > g->ms_cap) {
+    if (g->ms_items) CU(cudaFree(g->ms_items));
+    if (g->ms_sc) CU(cudaFree(g->ms_sc));
+    g->ms_items = nullptr;
+    g->ms_sc = nullptr;
+    CU(cudaMalloc(&g->ms_items, sizeof(u64) * (size_t)K * cap));
+    CU(cudaMalloc(&g->ms_sc, sizeof(SlotCtl) * K));
+    CU(cudaMemsetAsync(g->ms_items, 0xFF, sizeof(u64) * (size_t)K * cap, s));
+    CU(cudaMemsetAsync(g->ms_sc, 0, sizeof(SlotCtl) * K, s));
+    g->ms_K = K;
+    g->ms_cap = cap;
+  }
+  MParams p;
+  p.rowc = g->rowc;
+  p.arcs = g->arcs;
+  p.D = g->ms_D;
+  p.Q = g->ms_Q;
+  p.ctl = g->ms_ctl;
+  p.sc = g->ms_sc;
+  p.items = g->ms_items;
+  p.stats = g->ms_stats;
+  p.V = (u32)g->V;
+  p.K = g->ms_K;
+  p.kmask = g->ms_K - 1;
+  p.cap = g->ms_cap;
+  p.delta_u = dp.delta_u;
+  p.inv_delta = dp.inv;
+  p.f32 = f32 ? 1u : 0u;
+  p.inf = f32 ? 0x7F800000u : 0xFFFFFFFFu;
+  int per_sm = 0;
+  const void* mk = f32 ? (const void*)k_ms_step<true> : (const void*)k_ms_step<false>;
+  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mk, MS_THREADS, 0));
+  if (per_sm < 1) return fail(SSSP_ERR_INTERNAL, "multi-source kernel cannot be resident");
+  if (g->p_ctas > 0) per_sm = std::min<int>(per_sm, (int)g->p_ctas);
+  const int grid = per_sm * g->num_sms;
+  std::vector<u32> src(MS_LANES);
+  for (i64 g0 = 0; g0 < n; g0 += MS_LANES) {
+    const u32 nn = (u32)std::min<i64>(MS_LANES, n - g0);
+    for (u32 l = 0; l < nn; ++l)
+      src[l] = g->h_old2new.empty() ? (u32)sources[g0 + l] : g->h_old2new[sources[g0 + l]];
+    CU(cudaMemcpyAsync(g->ms_src, src.data(), sizeof(u32) * nn, cudaMemcpyHostToDevice, s));
+    k_ms_init<<<grid_for(g->V * (MS_LANES / 4)), 256, 0, s>>>(g->ms_D, g->ms_Q, g->V, p.inf);
+    k_ms_seed<<<1, 32, 0, s>>>(p, g->ms_src, nn);
+    CU(cudaGetLastError());
+    cudaEvent_t e0, e1;
+    for (int i = 0; i < 2; ++i) {
+      cudaEvent_t e;
+      if (g->ev_pool.empty()) {
+        CU(cudaEventCreate(&e));
+      } else {
+        e = g->ev_pool.back();
+        g->ev_pool.pop_back();
+      }
+      (i ? e1 : e0) = e;
+    }
+    g->ev_pending.emplace_back(e0, e1);
+    CU(cudaEventRecord(e0, s));
+    void* args[] = {&p};
+    CU(cudaLaunchCooperativeKernel(mk, dim3(grid), dim3(MS_THREADS), args, 0, s));
+    CU(cudaEventRecord(e1, s));
+    k_ms_output<<<grid_for(g->V), 256, 0, s>>>(g->ms_D, g->old2new, g->V, nn, (u32*)out_dev + (size_t)g0 * ld, ld);
+    CU(cudaGetLastError());
+    CU(cudaStreamSynchronize(s));  // the source buffer is reused by the next group
+  }
+  MCtl c;
+  CU(cudaMemcpyAsync(&c, g->ms_ctl, sizeof c, cudaMemcpyDeviceToHost, s));
+  CU(cudaStreamSynchronize(s));
+  if (c.err & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_multi_stats(sssp_graph_t g, uint64_t* out, int64_t n) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out || n < 0) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad output");
+  if (!g->ms_stats) return fail(SSSP_ERR_INVALID_STATE, "no sssp_run_multi yet");
+  DeviceGuard dg(g->device);
+  unsigned long long h[MST_N];
+  MCtl c;
+  CU(cudaMemcpyAsync(h, g->ms_stats, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaMemcpyAsync(&c, g->ms_ctl, sizeof c, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaStreamSynchronize(g->stream));
+  const uint64_t v[7] = {h[MST_UPDATES], h[MST_ARCS], h[MST_EXPAND], h[MST_STALE], h[MST_CHUNKS], c.buckets, c.rescans};
+  for (int64_t i = 0; i < n && i < 7; ++i) out[i] = v[i];
   return SSSP_OK;
 }
 

@@ -455,3 +455,65 @@ def test_adaptive_delta_follows_eq1(sssp, mode, reading):
     assert len(set(r["mode"] for r in recs)) > 1, "Delta never changed"
     # C_i counts each settled vertex once (the last bucket closes without a record)
     assert sum(C) <= int((exp != INF).sum())
+
+
+# --------------------------------------- batched multi-source (NEXT-4) ----
+def _multi(sssp, G, srcs, delta, V, f32):
+    import torch
+
+    out = torch.empty((len(srcs), V), dtype=torch.float32 if f32 else torch.int32, device="cuda")
+    G.run_multi(srcs, delta, out)
+    return out.cpu().numpy().view(np.float32 if f32 else np.uint32)
+
+
+@pytest.mark.parametrize("wt,deltas", [("u32", (1, 16, 64, float("inf"))), ("f32", (0.02, 0.1, float("inf")))])
+@pytest.mark.parametrize("flags", [3, 0])
+def test_multi_source_parity(sssp, wt, deltas, flags):
+    """sssp_run_multi: 40 sources (a full 32-lane group + a partial one, with a
+    repeated source) bit-exact against per-source Dijkstra."""
+    g = gen.kronecker(12, 16, seed=55, weights=wt)
+    srcs = [int(s) for s in gen.sample_sources(g, 39, seed=21)]
+    srcs.append(srcs[3])
+    exp = np.stack([oracle.dijkstra(g.row, g.col, g.w, s) for s in srcs])
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if flags:
+            G.reorder(flags)
+        for d in deltas:
+            got = _multi(sssp, G, srcs, d, g.V, wt == "f32")
+            for i in range(len(srcs)):
+                assert_same(got[i], exp[i], f"multi {wt} flags={flags} delta={d} src#{i}={srcs[i]}")
+            st = G.multi_stats()
+            assert st["expansions"] > 0 and st["arcs"] > 0
+
+
+def test_multi_source_grid_and_hubs(sssp):
+    """Many buckets (grid), ring-horizon rescans (delta 1 with weights up to
+    100), and adjacencies split into 256-arc items (two 30000-arc hubs)."""
+    g = gen.grid(300, 200, p=0.2, seed=5)
+    srcs = [int(s) for s in gen.sample_sources(g, 8, seed=4)]
+    exp = np.stack([oracle.dijkstra(g.row, g.col, g.w, s) for s in srcs])
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        for d in (1, 400):
+            got = _multi(sssp, G, srcs, d, g.V, False)
+            for i in range(len(srcs)):
+                assert_same(got[i], exp[i], f"grid multi delta={d} src={srcs[i]}")
+        assert G.multi_stats()["buckets"] > 50
+    n = 30000
+    rng = np.random.default_rng(5)
+    arcs = []
+    for i in range(1, n + 1):
+        w = int(rng.integers(1, 100))
+        arcs += [(0, i, w), (i, 0, w), (1, i, w + 1), (i, 1, w + 1)]
+    row, col, w = csr_from_arcs(n + 1, arcs)
+    srcs = [0, 1, 5, 77, 29999]
+    exp = np.stack([oracle.dijkstra(row, col, w, s) for s in srcs])
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        for d in (1, 10):
+            got = _multi(sssp, G, srcs, d, n + 1, False)
+            for i in range(len(srcs)):
+                assert_same(got[i], exp[i], f"hub multi delta={d} src={srcs[i]}")
+            assert G.multi_stats()["split_items"] > 0
+            if d == 1:
+                assert G.multi_stats()["rescans"] >= 0
