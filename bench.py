@@ -31,6 +31,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 PAPER_V100 = {"C3": 16.78, "C4": 20.16}  # GTEPS, PAPER Fig. 11, context only
+MULTI_DELTA = {"C1": 256, "C3": 0.4, "C4": 256, "C5": 256}  # sssp_run_multi default Delta per config
 METRIC = "SSSP GTEPS (m/time) at 1 GPU; multi-source GTEPS at 1/2/4/8 B200; HBM GB/s"
 
 
@@ -245,6 +246,10 @@ def main():
         reorder_ms = G.stats()["reorder_ms"]
     inf = 0x7F800000 if g.wtype == "f32" else 0xFFFFFFFF
     if args.multi:
+        # swept on B200 (profiles/r01c/multi_delta_sweep.txt): the batched kernel prefers wide buckets
+        if args.delta is None:
+            delta = MULTI_DELTA.get(args.config, delta)
+            desc, _ = workload_desc(args.config, cfg, delta, reorder)
         return bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, stream,
                            reorder, reorder_ms, t_gen, inf)
 

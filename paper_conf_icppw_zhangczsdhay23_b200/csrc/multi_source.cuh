@@ -18,8 +18,8 @@
 // barrier when the current one is quiescent (pend == 0), like phase 3.
 //
 // Improvement protocol (no lost wake-ups): the improver does atomicMin(D),
-// fence, atomicMin(Q[v], bucket) and pushes v iff Q dropped; the expander
-// does atomicExch(Q[v], NONE), fence, then reads D[v]. Either the expander
+// __syncwarp, a release atomicMin(Q[v], bucket) and pushes v iff Q dropped; the
+// expander does an acquire atomicExch(Q[v], NONE), then reads D[v]. Either the expander
 // sees the new D, or the improver sees Q == NONE and queues v again.
 #pragma once
 #include "delta_step.cuh"
@@ -34,7 +34,10 @@ constexpr u32 MS_CHUNK = 256;  // arcs per work item: longer adjacencies are spl
 #define SSSP_MS_U 2
 #endif
 constexpr int MS_U = SSSP_MS_U;  // warp steps (4 arcs each) whose rows are in flight together
-constexpr u32 MS_CLAIM = 4;    // queue items per warp claim
+#ifndef SSSP_MS_CLAIM
+#define SSSP_MS_CLAIM 16
+#endif
+constexpr u32 MS_CLAIM = SSSP_MS_CLAIM;  // queue items per warp claim
 constexpr u32 MS_PB = 96;      // staged pushes per warp
 
 enum : u32 { MS_RUN = 0, MS_DONE = 2, MS_RESCAN_CLEAR = 3, MS_RESCAN_FILL = 4 };
@@ -63,9 +66,16 @@ struct MParams {
   u32 f32, inf;     // weight type; INF bits
 };
 
+#ifndef SSSP_MS_DEFER
+#define SSSP_MS_DEFER 0  // 1: D updates fire-and-forget (red.min), Q publications batched per warp (measured slower)
+#endif
+constexpr u32 MS_CB = 64;  // deferred (bucket << 32 | v) Q publications per warp
+
 struct MSmem {
   u64 pb[MS_WARPS][MS_PB];
   u32 pb_n[MS_WARPS];
+  u64 cb[MS_WARPS][MS_CB];
+  u32 cb_n[MS_WARPS];
   unsigned long long st[MST_N];
   u32 mode, cur, lim, base;
 };
@@ -126,7 +136,78 @@ __device__ __forceinline__ uint4 ms_probe4(const u32* a, bool pred) {
   return v;
 }
 
-__device__ __forceinline__ void ms_fence() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// Q[v] publication: the improver's min is a release (the warp's D atomics,
+// ordered before it by __syncwarp, become visible with it; SASS: MEMBAR.ALL.GPU
+// + ATOM, no L1 invalidate), the expander's exchange an acquire (ATOM +
+// CCTL.IVALL), so an expander that sees the new Q value also sees the new D.
+#ifndef SSSP_MS_FENCE
+#define SSSP_MS_FENCE 1
+#endif
+// Predicated atomicMin; returns 0 (so "nd < old" is false) when !pred.
+__device__ __forceinline__ u32 ms_atomic_min(u32* a, u32 v, bool pred) {
+  u32 old;
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n mov.b32 %0, 0;\n"
+      " @q atom.relaxed.gpu.global.min.u32 %0, [%1], %2;\n}"
+      : "=r"(old)
+      : "l"(a), "r"(v), "r"((u32)pred)
+      : "memory");
+  return old;
+}
+
+__device__ __forceinline__ u32 ms_q_min_release(u32* a, u32 v) {
+  u32 old;
+#if SSSP_MS_FENCE
+  asm volatile("atom.release.gpu.global.min.u32 %0, [%1], %2;" : "=r"(old) : "l"(a), "r"(v) : "memory");
+#else
+  old = atomicMin(a, v);
+#endif
+  return old;
+}
+__device__ __forceinline__ u32 ms_q_take_acquire(u32* a) {
+  u32 old;
+  asm volatile("atom.acquire.gpu.global.exch.b32 %0, [%1], %2;" : "=r"(old) : "l"(a), "r"(NONE) : "memory");
+  return old;
+}
+
+__device__ __forceinline__ void ms_red_min(u32* a, u32 v, bool pred) {
+  asm volatile(
+      "{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n"
+      " @q red.relaxed.gpu.global.min.u32 [%0], %1;\n}" ::"l"(a), "r"(v), "r"((u32)pred)
+      : "memory");
+}
+
+// Stage this warp's queue pushes (lanes with push) for ms_flush.
+__device__ __forceinline__ void ms_stage_pushes(const MParams& p, MSmem& sm, bool push, u32 key, u32 v) {
+  const u32 m = __ballot_sync(SSSP_FULL_MASK, push);
+  if (m) {
+    const u32 w = threadIdx.x >> 5;
+    if (sm.pb_n[w] + __popc(m) > MS_PB) ms_flush(p, sm);
+    if (push) sm.pb[w][sm.pb_n[w] + __popc(m & lanemask_lt())] = ((u64)key << 32) | v;
+    __syncwarp();
+    if (lane_id() == 0) sm.pb_n[w] += __popc(m);
+    __syncwarp();
+  }
+}
+
+// Deferred Q publications of warp w: Q[v] = min(Q[v], bucket) as release
+// atomics (after __syncwarp, so every red.min the warp issued before is
+// visible to the acquiring expander), queueing v where Q dropped.
+__device__ __noinline__ void ms_publish(const MParams p, MSmem& sm) {
+  const u32 lane = lane_id(), w = threadIdx.x >> 5;
+  const u32 n = sm.cb_n[w];
+  __syncwarp();
+  for (u32 i0 = 0; i0 < n; i0 += 32) {
+    const u32 i = i0 + lane;
+    const u64 e = i < n ? sm.cb[w][i] : ~0ULL;
+    const u32 key = (u32)(e >> 32), v = (u32)e;
+    const bool push = i < n && ms_q_min_release(p.Q + v, key) > key;
+    ms_stage_pushes(p, sm, push, key, v);
+  }
+  __syncwarp();
+  if (lane == 0) sm.cb_n[w] = 0;
+  __syncwarp();
+}
 
 // Relax arcs [b, e) of vertex u for every finite source of the group. Lane l
 // holds sources 4*(l&7) .. 4*(l&7)+3 (du = D[u][those]); the 8 lanes of
@@ -138,9 +219,11 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
   const u32 lane = lane_id(), grp = lane >> 3, sub = lane & 7, cur = sm.cur;
   const u64 pol_stream = policy_evict_first();
   bool ovf = false;
+  uint2 arc_next = ld_arc(p.arcs + b + lane, b + lane < e, pol_stream);
   for (u32 a0 = b; a0 < e; a0 += 32) {
     const u32 na = min(32u, e - a0);
-    const uint2 arc = ld_arc(p.arcs + a0 + lane, lane < na, pol_stream);
+    const uint2 arc = arc_next;  // this chunk's arcs; the next chunk's load starts now
+    arc_next = ld_arc(p.arcs + a0 + 32 + lane, a0 + 32 + lane < e, pol_stream);
     for (u32 t = 0; t < na; t += 4 * MS_U) {
       u32 dst[MS_U], nd[MS_U][4];
       uint4 pr[MS_U];
@@ -165,6 +248,10 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
         pr[k] = ms_probe4(p.D + (u64)dst[k] * MS_LANES + 4 * sub, ok[k]);
       }
       u32 mn[MS_U];
+#if SSSP_MS_DEFER
+      // Alg. 1 l.2-3 as a fire-and-forget red.min wherever the probe says the
+      // candidate is smaller; the candidate counts as an update (it may lose to
+      // a concurrent smaller one: then v is only queued once too often).
 #pragma unroll
       for (int k = 0; k < MS_U; ++k) {
         const u32 pv[4] = {pr[k].x, pr[k].y, pr[k].z, pr[k].w};
@@ -172,15 +259,34 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
         mn[k] = NONE;
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
-          if (ok[k] && nd[k][c] < pv[c]) {  // Alg. 1 l.2, then l.3
-            const u32 old = atomicMin(row + c, nd[k][c]);
-            if (nd[k][c] < old) {
-              ++c_upd;
-              mn[k] = min(mn[k], nd[k][c]);
-            }
-          }
+          const bool want = ok[k] && nd[k][c] < pv[c];
+          ms_red_min(row + c, nd[k][c], want);
+          c_upd += want;
+          mn[k] = want ? min(mn[k], nd[k][c]) : mn[k];
         }
       }
+#else
+      // all 4 * MS_U atomics in flight before any result is consumed
+      u32 old[MS_U][4];
+#pragma unroll
+      for (int k = 0; k < MS_U; ++k) {
+        const u32 pv[4] = {pr[k].x, pr[k].y, pr[k].z, pr[k].w};
+        u32* row = p.D + (u64)dst[k] * MS_LANES + 4 * sub;
+#pragma unroll
+        for (int c = 0; c < 4; ++c)  // Alg. 1 l.2, then l.3 (0 when not issued)
+          old[k][c] = ms_atomic_min(row + c, nd[k][c], ok[k] && nd[k][c] < pv[c]);
+      }
+#pragma unroll
+      for (int k = 0; k < MS_U; ++k) {
+        mn[k] = NONE;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          const bool imp = nd[k][c] < old[k][c];
+          c_upd += imp;
+          mn[k] = imp ? min(mn[k], nd[k][c]) : mn[k];
+        }
+      }
+#endif
       // smallest improved distance of each arc over its 32 sources (8 lanes)
 #pragma unroll
       for (int k = 0; k < MS_U; ++k) {
@@ -200,23 +306,24 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
           my_key = max(F32 ? ms_bucket_f(p, m) : m / p.delta_u, cur);
         }
       }
+#if SSSP_MS_DEFER
+      const u32 cm = __ballot_sync(SSSP_FULL_MASK, my_key != NONE);
+      if (cm) {  // defer: one release fence per batch of publications (ms_publish)
+        const u32 w = threadIdx.x >> 5;
+        if (sm.cb_n[w] + __popc(cm) > MS_CB) ms_publish(p, sm);
+        if (my_key != NONE) sm.cb[w][sm.cb_n[w] + __popc(cm & lanemask_lt())] = ((u64)my_key << 32) | my_dst;
+        __syncwarp();
+        if (lane == 0) sm.cb_n[w] += __popc(cm);
+        __syncwarp();
+      }
+#else
       if (__any_sync(SSSP_FULL_MASK, my_key != NONE)) {
         __syncwarp();
         bool push = false;
-        if (my_key != NONE) {
-          ms_fence();  // the D atomics above happen-before the Q update (see header)
-          push = atomicMin(p.Q + my_dst, my_key) > my_key;
-        }
-        const u32 m = __ballot_sync(SSSP_FULL_MASK, push);
-        if (m) {
-          const u32 w = threadIdx.x >> 5;
-          if (sm.pb_n[w] + __popc(m) > MS_PB) ms_flush(p, sm);
-          if (push) sm.pb[w][sm.pb_n[w] + __popc(m & lanemask_lt())] = ((u64)my_key << 32) | my_dst;
-          __syncwarp();
-          if (lane == 0) sm.pb_n[w] += __popc(m);
-          __syncwarp();
-        }
+        if (my_key != NONE) push = ms_q_min_release(p.Q + my_dst, my_key) > my_key;
+        ms_stage_pushes(p, sm, push, my_key, my_dst);
       }
+#endif
     }
   }
   if (!F32 && ovf) atomicOr(&p.ctl->err, ERR_OVERFLOW);
@@ -277,8 +384,7 @@ __device__ void ms_bucket_run(const MParams& p, MSmem& sm) {
       } else {
         u32 x = 0;
         if (lane == 0) {
-          x = atomicExch(p.Q + v, NONE);
-          ms_fence();
+          x = ms_q_take_acquire(p.Q + v);
         }
         x = __shfl_sync(SSSP_FULL_MASK, x, 0);
         __syncwarp();
@@ -310,6 +416,9 @@ __device__ void ms_bucket_run(const MParams& p, MSmem& sm) {
       c_arcs += en - b;
       ms_relax<F32>(p, sm, b, en, du, c_upd);
     }
+#if SSSP_MS_DEFER
+    if (sm.cb_n[threadIdx.x >> 5]) ms_publish(p, sm);
+#endif
     if (sm.pb_n[threadIdx.x >> 5]) ms_flush(p, sm);  // publish before completing
     if (lane == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);
   }
@@ -441,7 +550,7 @@ template <bool F32>
 __global__ void __launch_bounds__(MS_THREADS, SSSP_MS_MINB) k_ms_step(MParams p) {
   __shared__ MSmem sm;
   if (threadIdx.x < MST_N) sm.st[threadIdx.x] = 0;
-  if (threadIdx.x < MS_WARPS) sm.pb_n[threadIdx.x] = 0;
+  if (threadIdx.x < MS_WARPS) sm.pb_n[threadIdx.x] = sm.cb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
     volatile MCtl* vc = p.ctl;
     sm.mode = vc->mode;
