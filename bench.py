@@ -439,6 +439,24 @@ def bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, 
     value = n_all * g.m / (t_ms * 1e-3) / 1e9
     ms = G.multi_stats()
     e2e = None
+    if not args.no_e2e and not args.profile and world > 1:
+        # every rank runs its whole shard through sssp_run_multi, rows gathered to rank 0 over
+        # NCCL, rank 0 copies them to pinned host memory; wall clock, max over ranks
+        from paper_conf_icppw_zhangczsdhay23_b200 import batch
+
+        pinned = torch.empty((len(sources), g.V), dtype=torch.int32).pin_memory() if rank == 0 else None
+        torch.distributed.barrier()
+        t0 = time.perf_counter()
+        rows = batch.run_sharded(G, sources, delta, dst=0, kernel="multi")
+        if rank == 0:
+            pinned.copy_(rows.view(torch.int32) if rows.dtype != torch.int32 else rows)
+        torch.distributed.barrier()
+        te = torch.tensor([time.perf_counter() - t0], device=tdev)
+        torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
+        e2e = {"value": round(len(sources) * g.m / float(te.item()) / 1e9, 4), "unit": "GTEPS",
+               "h2d_bytes_per_step": 8 * len(sources), "d2h_bytes_per_step": 4 * g.V * len(sources),
+               "note": "one step = the whole source batch: each rank runs its shard (sssp_run_multi), NCCL "
+                       "gather of all rows to rank 0, copy to pinned host; wall clock, max over ranks"}
     if not args.no_e2e and not args.profile and world == 1:
         grp = groups[0]
         pinned = torch.empty((len(grp), g.V), dtype=torch.int32).pin_memory()

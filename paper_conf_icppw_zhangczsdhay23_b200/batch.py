@@ -60,9 +60,12 @@ def gather_rows(local_rows, n_sources: int, dst: int = 0, group=None):
     return out
 
 
-def run_sharded(graph, sources, delta, dst: int = 0, group=None):
+def run_sharded(graph, sources, delta, dst: int = 0, group=None, kernel: str = "per_source"):
     """Run this rank's shard of ``sources`` on ``graph`` (a paper_conf...Graph on
-    this rank's GPU) and gather all distance rows to ``dst``."""
+    this rank's GPU) and gather all distance rows to ``dst``. ``kernel``:
+    "per_source" = one persistent Delta-stepping launch per source
+    (``sssp_run_batch``), "multi" = 32 sources per launch (``sssp_run_multi``,
+    NEXT-4). Both give identical rows."""
     import torch
     import torch.distributed as dist
 
@@ -71,7 +74,9 @@ def run_sharded(graph, sources, delta, dst: int = 0, group=None):
     mine = shard_sources(sources, rank, world)
     dtype = torch.float32 if graph.f32 else torch.int32
     rows = torch.empty((max(len(mine), 1), graph.V), dtype=dtype, device=f"cuda:{graph.device}")
+    if kernel not in ("per_source", "multi"):
+        raise ValueError(f"unknown kernel {kernel!r}")
     if len(mine):
-        graph.run_batch(mine, delta, rows, graph.V)
+        (graph.run_multi if kernel == "multi" else graph.run_batch)(mine, delta, rows, graph.V)
     torch.cuda.synchronize(graph.device)
     return gather_rows(rows[: len(mine)] if len(mine) else rows[:0], len(sources), dst, group)
