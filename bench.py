@@ -31,7 +31,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 PAPER_V100 = {"C3": 16.78, "C4": 20.16}  # GTEPS, PAPER Fig. 11, context only
-MULTI_DELTA = {"C1": 256, "C3": 0.4, "C4": 256, "C5": 256}  # sssp_run_multi default Delta per config
+MULTI_DELTA = {"C1": 64, "C3": 0.1, "C4": 4, "C5": 2}  # sssp_run_multi default Delta (profiles/r01c/multi_delta_sweep.txt)
 METRIC = "SSSP GTEPS (m/time) at 1 GPU; multi-source GTEPS at 1/2/4/8 B200; HBM GB/s"
 
 

@@ -185,7 +185,7 @@ typedef enum {
                                       for buckets with >= value settled entries; smaller
                                       buckets (and -1 = never) relax heavy arcs through the
                                       phase-1 vertex bins [-1] */
-    SSSP_PARAM_ADAPTIVE_DELTA = 8  /* NEXT-1, Eq. (1)-(2) P:1006-1028 (Alg. 2 l.11): 0 fixed
+    SSSP_PARAM_ADAPTIVE_DELTA = 8, /* NEXT-1, Eq. (1)-(2) P:1006-1028 (Alg. 2 l.11): 0 fixed
                                       Delta; 1 Delta_i = Delta_{i-1} + eps_i (Eq. (2) as
                                       printed); 2 Delta_i = Delta_0 + eps_i (Fig. 6 text,
                                       P:1033-1037). eps_i from the converged-vertex and thread
@@ -193,6 +193,12 @@ typedef enum {
                                       Delta_i clamped to [Delta_0/4, 4 Delta_0]. The delta of
                                       sssp_run is Delta_0. Distances do not change (Delta-
                                       stepping is exact for every Delta) [0] */
+    SSSP_PARAM_MULTI_ALIGN = 9     /* sssp_run_multi: 1 orders the queue by distance + (M -
+                                      d(hub, source)) per source, so the 32 wavefronts that all
+                                      pass through the highest-degree vertex reach each vertex in
+                                      about the same bucket (one SSSP from that vertex per graph
+                                      and Delta, which replaces the last sssp_run result); 0 by
+                                      plain distance. Results are identical [1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

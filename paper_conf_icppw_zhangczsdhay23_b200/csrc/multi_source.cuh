@@ -60,6 +60,7 @@ struct MParams {
   SlotCtl* sc;        // [K]
   u64* items;         // [K * cap]: v, or (chunk << 32 | CHUNK_FLAG | v)
   unsigned long long* stats;  // [MST_N]
+  const u32* shift;           // [32] per-source queue-key shift (lane alignment, see ms_relax)
   u32 V, K, kmask, cap;
   u32 delta_u;      // u32: integer Delta
   float inv_delta;  // f32: fl32(1 / Delta)
@@ -209,13 +210,25 @@ __device__ __noinline__ void ms_publish(const MParams p, MSmem& sm) {
   __syncwarp();
 }
 
+// Queue keys use "aligned time" nd + shift[lane] instead of nd: the host
+// sets shift[l] = M - d(hub, source l) (M = the largest such distance), so the
+// 32 sources' wavefronts, which all pass through the hubs, reach a vertex in
+// about the same bucket and it is expanded about once for all of them. Any
+// key is correct (label-correcting); the shift only orders the work.
+template <bool F32>
+__device__ __forceinline__ u32 ms_time(u32 nd, u32 sh) {
+  if (F32) return __float_as_uint(__fadd_rn(__uint_as_float(nd), __uint_as_float(sh)));
+  const u64 t = (u64)nd + sh;
+  return t >= (u64)NONE ? NONE - 1 : (u32)t;
+}
+
 // Relax arcs [b, e) of vertex u for every finite source of the group. Lane l
 // holds sources 4*(l&7) .. 4*(l&7)+3 (du = D[u][those]); the 8 lanes of
 // group l>>3 relax one arc together, so a warp step covers 4 arcs and each
 // probe instruction reads four whole 128-byte rows.
 template <bool F32>
 __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32 e, const u32 (&du)[4],
-                                         u32& c_upd) {
+                                         const u32 (&sh)[4], u32& c_upd) {
   const u32 lane = lane_id(), grp = lane >> 3, sub = lane & 7, cur = sm.cur;
   const u64 pol_stream = policy_evict_first();
   bool ovf = false;
@@ -262,7 +275,7 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
           const bool want = ok[k] && nd[k][c] < pv[c];
           ms_red_min(row + c, nd[k][c], want);
           c_upd += want;
-          mn[k] = want ? min(mn[k], nd[k][c]) : mn[k];
+          mn[k] = want ? min(mn[k], ms_time<F32>(nd[k][c], sh[c])) : mn[k];
         }
       }
 #else
@@ -283,7 +296,7 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
         for (int c = 0; c < 4; ++c) {
           const bool imp = nd[k][c] < old[k][c];
           c_upd += imp;
-          mn[k] = imp ? min(mn[k], nd[k][c]) : mn[k];
+          mn[k] = imp ? min(mn[k], ms_time<F32>(nd[k][c], sh[c])) : mn[k];
         }
       }
 #endif
@@ -413,8 +426,10 @@ __device__ void ms_bucket_run(const MParams& p, MSmem& sm) {
       }
       const uint4 d4 = __ldcg(reinterpret_cast<const uint4*>(p.D + (u64)v * MS_LANES) + (lane & 7));
       const u32 du[4] = {d4.x, d4.y, d4.z, d4.w};
+      const uint4 s4 = __ldg(reinterpret_cast<const uint4*>(p.shift) + (lane & 7));
+      const u32 sh[4] = {s4.x, s4.y, s4.z, s4.w};
       c_arcs += en - b;
-      ms_relax<F32>(p, sm, b, en, du, c_upd);
+      ms_relax<F32>(p, sm, b, en, du, sh, c_upd);
     }
 #if SSSP_MS_DEFER
     if (sm.cb_n[threadIdx.x >> 5]) ms_publish(p, sm);

@@ -68,7 +68,9 @@ struct sssp_graph_s {
   SlotCtl* ms_sc = nullptr;
   MCtl* ms_ctl = nullptr;
   unsigned long long* ms_stats = nullptr;
-  u32* ms_src = nullptr;   // [32]
+  u32* ms_src = nullptr;   // [32] sources, then [32] key shifts
+  std::vector<u32> h_hubdist;  // distances from the max-degree vertex (lane alignment)
+  u32 hubdist_bits = 0xFFFFFFFFu;
   u32 ms_K = 0, ms_cap = 0;
   u32* out_tmp = nullptr;  // [V] staging for sssp_distances into pageable host memory
   unsigned long long* stats = nullptr;
@@ -87,7 +89,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -308,6 +310,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       if (v < 0 || v > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "adaptive delta is 0, 1 or 2");
       g->p_adapt = v;
       return SSSP_OK;
+    case SSSP_PARAM_MULTI_ALIGN:
+      if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "multi align is 0 or 1");
+      g->p_align = v;
+      return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
       g->p_claim = v;
@@ -451,6 +457,7 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   g->heavy_valid = false;
   g->rowc_valid = false;
   g->rowc_lv_valid = false;
+  g->hubdist_bits = 0xFFFFFFFFu;
   g->have_result = false;
   g->reorder_timed = true;
   return SSSP_OK;
@@ -819,7 +826,7 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
     CU(cudaMalloc(&g->ms_ctl, sizeof(MCtl)));
     CU(cudaMemsetAsync(g->ms_ctl, 0, sizeof(MCtl), s));
     CU(cudaMalloc(&g->ms_stats, sizeof(unsigned long long) * MST_N));
-    CU(cudaMalloc(&g->ms_src, sizeof(u32) * MS_LANES));
+    CU(cudaMalloc(&g->ms_src, sizeof(u32) * 2 * MS_LANES));
   }
   if (K > g->ms_K || cap > g->ms_cap) {
     if (g->ms_items) CU(cudaFree(g->ms_items));
@@ -842,6 +849,7 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
   p.sc = g->ms_sc;
   p.items = g->ms_items;
   p.stats = g->ms_stats;
+  p.shift = g->ms_src + MS_LANES;
   p.V = (u32)g->V;
   p.K = g->ms_K;
   p.kmask = g->ms_K - 1;
@@ -856,12 +864,58 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
   if (per_sm < 1) return fail(SSSP_ERR_INTERNAL, "multi-source kernel cannot be resident");
   if (g->p_ctas > 0) per_sm = std::min<int>(per_sm, (int)g->p_ctas);
   const int grid = per_sm * g->num_sms;
-  std::vector<u32> src(MS_LANES);
+  if (g->p_align && g->hubdist_bits != dp.delta_bits) {
+    // Lane alignment: distances from the highest-degree vertex (one single-source run,
+    // cached per graph; it replaces the last sssp_run result).
+    u32 hub = 0;
+    if (g->h_old2new.empty()) {
+      std::vector<long long> rp(g->V + 1);
+      std::vector<longlong2> tmp(g->V + 1);
+      CU(cudaMemcpyAsync(tmp.data(), g->rowp, sizeof(longlong2) * (g->V + 1), cudaMemcpyDeviceToHost, s));
+      CU(cudaStreamSynchronize(s));
+      long long best = -1;
+      for (i64 v = 0; v < g->V; ++v)
+        if (tmp[v + 1].x - tmp[v].x > best) best = tmp[v + 1].x - tmp[v].x, hub = (u32)v;
+    }  // degree-sorted (PRO): internal id 0 has the highest degree
+    DeltaParams dh = dp;
+    dh.ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
+    g->have_result = false;
+    if ((st = launch_run(g, hub, dh, false))) return st;
+    g->h_hubdist.resize(g->V);
+    CU(cudaMemcpyAsync(g->h_hubdist.data(), g->dist, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    g->hubdist_bits = dp.delta_bits;
+  }
+  std::vector<u32> src(2 * MS_LANES, 0u);
   for (i64 g0 = 0; g0 < n; g0 += MS_LANES) {
     const u32 nn = (u32)std::min<i64>(MS_LANES, n - g0);
     for (u32 l = 0; l < nn; ++l)
       src[l] = g->h_old2new.empty() ? (u32)sources[g0 + l] : g->h_old2new[sources[g0 + l]];
-    CU(cudaMemcpyAsync(g->ms_src, src.data(), sizeof(u32) * nn, cudaMemcpyHostToDevice, s));
+    // key shift of lane l: M - d(hub, source l) (0 for unreachable sources / alignment off)
+    std::fill(src.begin() + MS_LANES, src.end(), 0u);
+    if (g->p_align && !g->h_hubdist.empty()) {
+      if (f32) {
+        float M = 0.f;
+        for (u32 l = 0; l < nn; ++l) {
+          float d;
+          memcpy(&d, &g->h_hubdist[src[l]], 4);
+          if (std::isfinite(d)) M = std::max(M, d);
+        }
+        for (u32 l = 0; l < nn; ++l) {
+          float d, sh;
+          memcpy(&d, &g->h_hubdist[src[l]], 4);
+          sh = std::isfinite(d) ? M - d : 0.f;
+          memcpy(&src[MS_LANES + l], &sh, 4);
+        }
+      } else {
+        u32 M = 0;
+        for (u32 l = 0; l < nn; ++l)
+          if (g->h_hubdist[src[l]] != 0xFFFFFFFFu) M = std::max(M, g->h_hubdist[src[l]]);
+        for (u32 l = 0; l < nn; ++l)
+          src[MS_LANES + l] = g->h_hubdist[src[l]] != 0xFFFFFFFFu ? M - g->h_hubdist[src[l]] : 0u;
+      }
+    }
+    CU(cudaMemcpyAsync(g->ms_src, src.data(), sizeof(u32) * 2 * MS_LANES, cudaMemcpyHostToDevice, s));
     k_ms_init<<<grid_for(g->V * (MS_LANES / 4)), 256, 0, s>>>(g->ms_D, g->ms_Q, g->V, p.inf);
     k_ms_seed<<<1, 32, 0, s>>>(p, g->ms_src, nn);
     CU(cudaGetLastError());

@@ -130,3 +130,32 @@ def test_c4_pro_properties(sssp):
         h_new = np.sum(mix(src_new.astype(np.uint64), ex["adj"].astype(np.uint64),
                                           ex["val"].astype(np.uint64)), dtype=np.uint64)
     assert h_ref == h_new
+
+
+@pytest.mark.parametrize("name,n_exact", [("C4", 1), ("C3", 1), ("C1", 4)])
+def test_multi_source_full_size(sssp, name, n_exact):
+    """sssp_run_multi at full size in the bench --multi launch configuration
+    (one 32-source group, bench.MULTI_DELTA): rows bit-exact against the oracle
+    for the first sources, the shortest-path certificate for the other rows of
+    u32 configs, and every row equal to the single-source kernel's result for
+    a sample of lanes (both paths must give the unique distances)."""
+    import torch
+
+    import bench
+
+    g = graph(name)
+    delta = bench.MULTI_DELTA[name]
+    srcs = [int(s) for s in gen.sample_sources(g, 32, seed=7)]
+    f32 = g.wtype == "f32"
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        out = torch.empty((32, g.V), dtype=torch.float32 if f32 else torch.int32, device="cuda")
+        G.run_multi(srcs, delta, out)
+        rows = out.cpu().numpy()
+        for i in range(n_exact):
+            check(rows[i], oracle.dijkstra(g.row, g.col, g.w, srcs[i]), f"{name} multi src={srcs[i]}")
+        if not f32:
+            for i in (5, 17, 31):
+                assert oracle.certificate(g.row, g.col, g.w, srcs[i], rows[i]) == -1, f"{name} multi cert lane {i}"
+        for i in (2, 9, 30):
+            check(rows[i], G.sssp(srcs[i], gen.CONFIGS[name]["delta"]).copy(), f"{name} multi vs single lane {i}")

@@ -20,6 +20,8 @@ srcs = gen.sample_sources(g, n, seed=7)
 m = g.m
 with sssp.Graph(g.row, g.col, g.w) as G:
     G.reorder()
+    if os.environ.get("MULTI_ALIGN") is not None:
+        G.set_param(sssp.SSSP_PARAM_MULTI_ALIGN, int(os.environ["MULTI_ALIGN"]))
     out = torch.empty((n, g.V), dtype=torch.int32, device="cuda")
     out2 = torch.empty_like(out)
     for d in deltas:
