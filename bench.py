@@ -498,8 +498,8 @@ def bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, 
                    "l2": "inputs larger than L2 (D rows %.2f GB, arcs %.2f GB > 126 MB L2); D re-initialised "
                          "every step" % (128 * g.V / 1e9, 8 * g.A / 1e9), "gen_s": round(t_gen, 1)},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": None, "peak_kind": peak_kind,
-                     "kernel": "k_ms_step (persistent, 32 sources)", "kernel_ms_avg": round(kt_avg, 4),
+                     "frac": round(achieved / peak, 4), "traffic": load_traffic(args.config + "_multi"),
+                     "peak_kind": peak_kind, "kernel": "k_ms_step (persistent, 32 sources)", "kernel_ms_avg": round(kt_avg, 4),
                      "kernel_share_of_step": round(kt_total / t_ms, 4), "alg_bytes_per_launch": int(b_alg)},
         "cpu_baseline": cpu,
         "e2e": e2e,
