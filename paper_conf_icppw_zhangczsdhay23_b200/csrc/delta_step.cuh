@@ -69,7 +69,7 @@ constexpr int IPT_MAX = IPT > IPT2 ? IPT : IPT2;
 #define SSSP_CLAIM_MINPART 64u  // take a partial batch once this many entries are ready ...
 #endif
 #ifndef SSSP_CLAIM_WAIT_NS
-#define SSSP_CLAIM_WAIT_NS 2000u  // ... or after waiting this long for a full one
+#define SSSP_CLAIM_WAIT_NS 200u  // ... or after waiting this long for a full one (2000: C2 -4 %, C1 -8 %)
 #endif
 constexpr u64 SENTINEL = ~0ULL;
 constexpr u32 NONE = 0xFFFFFFFFu;

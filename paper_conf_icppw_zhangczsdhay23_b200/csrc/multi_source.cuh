@@ -29,7 +29,10 @@ namespace sssp {
 constexpr int MS_LANES = 32;
 constexpr int MS_THREADS = 256;
 constexpr int MS_WARPS = MS_THREADS / 32;
-constexpr u32 MS_CHUNK = 256;  // arcs per work item: longer adjacencies are split
+#ifndef SSSP_MS_CHUNK
+#define SSSP_MS_CHUNK 256
+#endif
+constexpr u32 MS_CHUNK = SSSP_MS_CHUNK;  // arcs per work item: longer adjacencies are split
 #ifndef SSSP_MS_U
 #define SSSP_MS_U 2
 #endif

@@ -517,3 +517,49 @@ def test_multi_source_grid_and_hubs(sssp):
             assert G.multi_stats()["split_items"] > 0
             if d == 1:
                 assert G.multi_stats()["rescans"] >= 0
+
+
+def test_multi_source_abi_errors(sssp):
+    import torch
+
+    g = gen.kronecker(8, 8, seed=3)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        with pytest.raises(sssp.SSSPError) as e:
+            G.multi_stats()
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+        out = torch.empty((4, g.V), dtype=torch.int32, device="cuda")
+        for bad_src in ([-1], [g.V]):
+            with pytest.raises(sssp.SSSPError) as e:
+                G.run_multi(bad_src, 16, out)
+            assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+        for bad in (0, -1, float("nan")):
+            with pytest.raises(sssp.SSSPError) as e:
+                G.run_multi([0], bad, out)
+            assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+        with pytest.raises(sssp.SSSPError) as e:
+            G.run_multi([0], 16, out, ld=g.V - 1)
+        assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+        G.run_multi([], 16, out)  # empty batch: no-op
+        # the hub run of the lane alignment replaces the last single-source result
+        G.sssp(0, 16)
+        G.run_multi([1, 2], 16, out)
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances()
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+        # alignment off: same rows
+        a = out[:2].cpu().numpy().copy()
+        G.set_param(sssp.SSSP_PARAM_MULTI_ALIGN, 0)
+        G.run_multi([1, 2], 16, out)
+        assert np.array_equal(a, out[:2].cpu().numpy())
+
+
+def test_multi_source_u32_overflow_reported(sssp):
+    import torch
+
+    big = 0x7FFFFFFF
+    row, col, w = csr_from_arcs(4, [(0, 1, big), (1, 0, big), (1, 2, big), (2, 1, big), (2, 3, 5), (3, 2, 5)])
+    with sssp.Graph(row, col, w) as G:
+        out = torch.empty((1, 4), dtype=torch.int32, device="cuda")
+        with pytest.raises(sssp.SSSPError) as e:
+            G.run_multi([0], 16, out)
+        assert e.value.status == sssp.SSSP_ERR_OVERFLOW
