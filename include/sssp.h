@@ -113,6 +113,19 @@ sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream);
  * i < n run sssp_run(sources[i], delta) and write the distances (original
  * order) to the DEVICE buffer out_dev + i*ld elements (ld >= V). sources is a
  * host array. Stream-ordered; no host synchronisation. */
+/* Asynchronous sssp_distances: the output gather of the last run (original
+ * ids, graph weight type) goes to one of two device staging buffers on the
+ * handle's stream, then a copy engine moves it to `out` on the handle's own
+ * output stream, so the transfer overlaps the next sssp_run. out: pinned host
+ * memory (cudaHostAlloc / torch pin_memory) or device memory (written on the
+ * handle's stream); valid, and not touched by the caller, until sssp_wait.
+ * Pageable memory: SSSP_ERR_INVALID_ARGUMENT. INVALID_STATE before a run. */
+sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memory where);
+
+/* Waits for every output enqueued by sssp_distances_async. (Run errors are
+ * reported by sssp_run itself, which waits for its own kernel.) */
+sssp_status sssp_wait(sssp_graph_t g);
+
 sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                            void* out_dev, int64_t ld);
 

@@ -56,6 +56,7 @@ EXPORTS = (
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
     "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile", "sssp_run_multi", "sssp_multi_stats",
+    "sssp_distances_async", "sssp_wait",
 )
 
 
@@ -85,6 +86,8 @@ _lib.sssp_last_error.restype = ctypes.c_char_p
 _lib.sssp_set_stream.argtypes = [_P, _P]
 _lib.sssp_run_batch.argtypes = [_P, _P, _I64, _D, _P, _I64]
 _lib.sssp_run_multi.argtypes = [_P, _P, _I64, _D, _P, _I64]
+_lib.sssp_distances_async.argtypes = [_P, _P, _I]
+_lib.sssp_wait.argtypes = [_P]
 _lib.sssp_multi_stats.argtypes = [_P, _P, _I64]
 _lib.sssp_get_stats.argtypes = [_P, ctypes.POINTER(sssp_stats)]
 _lib.sssp_export_csr.argtypes = [_P, _D, _P, _P, _P, _P]
@@ -106,7 +109,7 @@ _lib.sssp_get_profile.argtypes = [_P, _P, _I]
 _lib.sssp_get_profile.restype = _I
 for _n in ("sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
            "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param",
-           "sssp_run_multi", "sssp_multi_stats"):
+           "sssp_run_multi", "sssp_multi_stats", "sssp_distances_async", "sssp_wait"):
     getattr(_lib, _n).restype = _I
 
 
@@ -182,6 +185,18 @@ def sssp_distances(h, out):
     p, kind = _ptr(out)
     _check(_lib.sssp_distances(h, p, kind), "sssp_distances")
     return out
+
+
+def sssp_distances_async(h, out):
+    """Enqueue the output of the last run into ``out`` (pinned host or CUDA
+    tensor) on the library's output stream; ``out`` is valid after sssp_wait."""
+    p, kind = _ptr(out)
+    _check(_lib.sssp_distances_async(h, p, kind), "sssp_distances_async")
+    return out
+
+
+def sssp_wait(h):
+    _check(_lib.sssp_wait(h), "sssp_wait")
 
 
 def sssp_destroy(h):
@@ -309,6 +324,14 @@ class Graph:
         if out is None:
             out = np.empty(self.V, dtype=np.float32 if self.f32 else np.uint32)
         return sssp_distances(self.h, out)
+
+    def distances_async(self, out):
+        """Stream the last run's distances into `out` (pinned host or CUDA tensor)
+        while the next run proceeds; read `out` only after wait()."""
+        return sssp_distances_async(self.h, out)
+
+    def wait(self):
+        sssp_wait(self.h)
 
     def sssp(self, source, delta, out=None):
         self.run(source, delta)

@@ -73,6 +73,14 @@ struct sssp_graph_s {
   u32 hubdist_bits = 0xFFFFFFFFu;
   u32 ms_K = 0, ms_cap = 0;
   u32* out_tmp = nullptr;  // [V] staging for sssp_distances into pageable host memory
+  // sssp_distances_async: the output gather writes a device staging buffer (fast, on
+  // the run stream), a copy engine moves it to the host on d2h while the next run computes
+  u32* stage[2] = {nullptr, nullptr};
+  int stage_next = 0;
+  bool stage_used[2] = {false, false};
+  cudaEvent_t ev_out[2] = {nullptr, nullptr};
+  cudaEvent_t ev_ran = nullptr;
+  cudaStream_t d2h = nullptr;
   unsigned long long* stats = nullptr;
   TraceEnt* trace = nullptr;
   u32 K_alloc = 0, cap_alloc = 0, hub_cap = 0;
@@ -234,7 +242,12 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   DeviceGuard dg(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
   else cudaDeviceSynchronize();
-  void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->xd, g->ctl, g->sc,
+  if (g->d2h) cudaStreamSynchronize(g->d2h);
+  for (auto& e : g->ev_out)
+    if (e) cudaEventDestroy(e);
+  if (g->ev_ran) cudaEventDestroy(g->ev_ran);
+  if (g->d2h) cudaStreamDestroy(g->d2h);
+  void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->stage[0], g->stage[1], g->xd, g->ctl, g->sc,
                   g->items, g->hub_items, g->p2o, g->rowc_lv, g->ms_D, g->ms_Q, g->ms_items, g->ms_sc, g->ms_ctl, g->ms_stats, g->ms_src, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -771,6 +784,54 @@ extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory whe
   CU(cudaGetLastError());
   if (staged) CU(cudaMemcpyAsync(out, g->out_tmp, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
   return check_run_errors(g);
+}
+
+extern "C" sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memory where) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+  if (where != SSSP_MEM_HOST && where != SSSP_MEM_DEVICE) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad memory kind");
+  if (!g->have_result) return fail(SSSP_ERR_INVALID_STATE, "no successful sssp_run since create/reorder");
+  DeviceGuard dg(g->device);
+  cudaStream_t s = g->stream;
+  if (where == SSSP_MEM_DEVICE) {  // a8 straight into the caller's device buffer
+    k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, (u32*)out);
+    CU(cudaGetLastError());
+    return SSSP_OK;
+  }
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, out) != cudaSuccess || pa.type != cudaMemoryTypeHost) {
+    cudaGetLastError();
+    return fail(SSSP_ERR_INVALID_ARGUMENT, "sssp_distances_async needs pinned host memory");
+  }
+  if (!g->d2h) {
+    CU(cudaStreamCreateWithFlags(&g->d2h, cudaStreamNonBlocking));
+    CU(cudaEventCreateWithFlags(&g->ev_ran, cudaEventDisableTiming));
+    for (auto& e : g->ev_out) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  const int j = g->stage_next;
+  g->stage_next ^= 1;
+  if (!g->stage[j]) CU(cudaMalloc(&g->stage[j], sizeof(u32) * g->V));
+  if (g->stage_used[j]) CU(cudaStreamWaitEvent(s, g->ev_out[j], 0));  // its previous copy is done
+  // a8 into the staging buffer (HBM speed, run stream), then the copy engine moves it to
+  // the host on d2h while the next sssp_run computes
+  k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, g->stage[j]);
+  CU(cudaGetLastError());
+  CU(cudaEventRecord(g->ev_ran, s));
+  CU(cudaStreamWaitEvent(g->d2h, g->ev_ran, 0));
+  CU(cudaMemcpyAsync(out, g->stage[j], sizeof(u32) * g->V, cudaMemcpyDeviceToHost, g->d2h));
+  CU(cudaEventRecord(g->ev_out[j], g->d2h));
+  g->stage_used[j] = true;
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_wait(sssp_graph_t g) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  DeviceGuard dg(g->device);
+  CU(cudaStreamSynchronize(g->stream));
+  if (g->d2h) CU(cudaStreamSynchronize(g->d2h));
+  return SSSP_OK;
 }
 
 extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,

@@ -563,3 +563,34 @@ def test_multi_source_u32_overflow_reported(sssp):
         with pytest.raises(sssp.SSSPError) as e:
             G.run_multi([0], 16, out)
         assert e.value.status == sssp.SSSP_ERR_OVERFLOW
+
+
+def test_distances_async_pipeline(sssp):
+    """sssp_distances_async overlaps step k's output with step k+1's run: every
+    pinned buffer ends with its own source's distances (oracle), errors of all
+    pageable memory is rejected."""
+    import torch
+
+    g = gen.kronecker(12, 16, seed=12)
+    srcs = [int(s) for s in gen.sample_sources(g, 6, seed=3)]
+    exp = [oracle.dijkstra(g.row, g.col, g.w, s) for s in srcs]
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances_async(torch.empty(g.V, dtype=torch.int32).pin_memory())
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+        bufs = [torch.empty(g.V, dtype=torch.int32).pin_memory() for _ in srcs]
+        dev = torch.empty(g.V, dtype=torch.int32, device="cuda")
+        for s, b in zip(srcs, bufs):
+            G.run(s, 16)
+            G.distances_async(b)
+        G.run(srcs[0], 16)
+        G.distances_async(dev)
+        G.wait()
+        for i, b in enumerate(bufs):
+            assert_same(b.numpy().view(np.uint32), exp[i], f"async src={srcs[i]}")
+        assert_same(dev.cpu().numpy().view(np.uint32), exp[0], "async device")
+        assert_same(G.distances(), exp[0], "sync after async")
+        with pytest.raises(sssp.SSSPError) as e:
+            G.distances_async(np.empty(g.V, dtype=np.uint32))
+        assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
