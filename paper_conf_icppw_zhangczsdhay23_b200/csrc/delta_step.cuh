@@ -38,7 +38,10 @@ namespace sssp {
 #ifndef SSSP_MINB
 #define SSSP_MINB 4  // persistent CTAs per SM the register budget is sized for
 #endif
-constexpr int DS_THREADS = 256;
+#ifndef SSSP_DS_THREADS
+#define SSSP_DS_THREADS 256
+#endif
+constexpr int DS_THREADS = SSSP_DS_THREADS;
 constexpr int DS_WARPS = DS_THREADS / 32;
 constexpr u32 BIN_WARP = 32;     // beta
 constexpr u32 BIN_CTA = 256;     // alpha

@@ -159,3 +159,28 @@ def test_multi_source_full_size(sssp, name, n_exact):
                 assert oracle.certificate(g.row, g.col, g.w, srcs[i], rows[i]) == -1, f"{name} multi cert lane {i}"
         for i in (2, 9, 30):
             check(rows[i], G.sssp(srcs[i], gen.CONFIGS[name]["delta"]).copy(), f"{name} multi vs single lane {i}")
+
+
+def test_c5_full_size_certificates(sssp):
+    """C5 (Kronecker scale 26, 2.1 G arcs, int64 row offsets) in both bench launch
+    configurations: one single-source run (config Delta) and one 32-source
+    sssp_run_multi group (bench.MULTI_DELTA), each checked with the complete
+    shortest-path certificate (u32 weights >= 1: d[s] = 0, every arc satisfied,
+    every reachable vertex tight on some arc, unreachable = no finite neighbour)."""
+    import torch
+
+    import bench
+
+    g = graph("C5")
+    srcs = [int(s) for s in gen.sample_sources(g, 32, seed=7)]
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        d = G.sssp(srcs[0], gen.CONFIGS["C5"]["delta"]).copy()
+        assert oracle.certificate(g.row, g.col, g.w, srcs[0], d) == -1, "C5 single-source certificate"
+        out = torch.empty((32, g.V), dtype=torch.int32, device="cuda")
+        G.run_multi(srcs, bench.MULTI_DELTA["C5"], out)
+        for i in (0, 13, 31):
+            row = out[i].cpu().numpy().view(np.uint32)
+            assert oracle.certificate(g.row, g.col, g.w, srcs[i], row) == -1, f"C5 multi certificate lane {i}"
+        assert np.array_equal(out[0].cpu().numpy().view(np.uint32), d.view(np.uint32))
+    _graphs.pop("C5", None)
