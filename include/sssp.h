@@ -206,12 +206,16 @@ typedef enum {
                                       Delta_i clamped to [Delta_0/4, 4 Delta_0]. The delta of
                                       sssp_run is Delta_0. Distances do not change (Delta-
                                       stepping is exact for every Delta) [0] */
-    SSSP_PARAM_MULTI_ALIGN = 9     /* sssp_run_multi: 1 orders the queue by distance + (M -
+    SSSP_PARAM_MULTI_ALIGN = 9,    /* sssp_run_multi: 1 orders the queue by distance + (M -
                                       d(hub, source)) per source, so the 32 wavefronts that all
                                       pass through the highest-degree vertex reach each vertex in
                                       about the same bucket (one SSSP from that vertex per graph
                                       and Delta, which replaces the last sssp_run result); 0 by
                                       plain distance. Results are identical [1] */
+    SSSP_PARAM_MULTI_HUB_DELAY = 10 /* sssp_run_multi on a degree-reordered graph: vertices
+                                      of degree > 1024 are queued this many buckets late, so
+                                      more of the 32 sources reach a hub before its (long)
+                                      adjacency is expanded; 0..16. Results are identical [0] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

@@ -47,6 +47,7 @@ SSSP_PARAM_SYNC = 6
 SSSP_PARAM_P2_EDGE_BALANCED = 7
 SSSP_PARAM_ADAPTIVE_DELTA = 8
 SSSP_PARAM_MULTI_ALIGN = 9
+SSSP_PARAM_MULTI_HUB_DELAY = 10
 
 INF_U32 = 0xFFFFFFFF
 

@@ -68,6 +68,8 @@ struct MParams {
   u32 delta_u;      // u32: integer Delta
   float inv_delta;  // f32: fl32(1 / Delta)
   u32 f32, inf;     // weight type; INF bits
+  u32 hub_ids;      // internal ids < hub_ids are high-degree vertices (PRO degree order) ...
+  u32 hub_delay;    // ... queued hub_delay buckets late, so more sources reach them first
 };
 
 #ifndef SSSP_MS_DEFER
@@ -319,7 +321,7 @@ __device__ __forceinline__ void ms_relax(const MParams& p, MSmem& sm, u32 b, u32
         const u32 d = __shfl_sync(SSSP_FULL_MASK, dst[k], src_lane);
         if ((lane >> 2) == (u32)k && m != NONE) {
           my_dst = d;
-          my_key = max(F32 ? ms_bucket_f(p, m) : m / p.delta_u, cur);
+          my_key = max(F32 ? ms_bucket_f(p, m) : m / p.delta_u, cur) + (d < p.hub_ids ? p.hub_delay : 0u);
         }
       }
 #if SSSP_MS_DEFER

@@ -97,7 +97,8 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0;
+  i64 hub_ids_cached = -1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -327,6 +328,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "multi align is 0 or 1");
       g->p_align = v;
       return SSSP_OK;
+    case SSSP_PARAM_MULTI_HUB_DELAY:
+      if (v < 0 || v > 16) return fail(SSSP_ERR_INVALID_ARGUMENT, "hub delay in [0,16]");
+      g->p_hub_delay = v;
+      return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
       g->p_claim = v;
@@ -471,6 +476,7 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   g->rowc_valid = false;
   g->rowc_lv_valid = false;
   g->hubdist_bits = 0xFFFFFFFFu;
+  g->hub_ids_cached = -1;
   g->have_result = false;
   g->reorder_timed = true;
   return SSSP_OK;
@@ -919,6 +925,21 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
   p.inv_delta = dp.inv;
   p.f32 = f32 ? 1u : 0u;
   p.inf = f32 ? 0x7F800000u : 0xFFFFFFFFu;
+  p.hub_ids = 0;
+  p.hub_delay = (u32)g->p_hub_delay;
+  if (g->p_hub_delay > 0 && !g->h_old2new.empty()) {  // degree-sorted ids: count degree > 1024
+    if (g->hub_ids_cached < 0) {
+      std::vector<longlong2> r(2);
+      u32 lo = 0, hi = (u32)g->V;  // first id with degree <= 1024 (degrees non-increasing)
+      while (lo < hi) {
+        const u32 mid = lo + (hi - lo) / 2;
+        CU(cudaMemcpy(r.data(), g->rowp + mid, 2 * sizeof(longlong2), cudaMemcpyDeviceToHost));
+        if (r[1].x - r[0].x > 1024) lo = mid + 1; else hi = mid;
+      }
+      g->hub_ids_cached = lo;
+    }
+    p.hub_ids = (u32)g->hub_ids_cached;
+  }
   int per_sm = 0;
   const void* mk = f32 ? (const void*)k_ms_step<true> : (const void*)k_ms_step<false>;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mk, MS_THREADS, 0));

@@ -22,6 +22,8 @@ with sssp.Graph(g.row, g.col, g.w) as G:
     G.reorder()
     if os.environ.get("MULTI_ALIGN") is not None:
         G.set_param(sssp.SSSP_PARAM_MULTI_ALIGN, int(os.environ["MULTI_ALIGN"]))
+    if os.environ.get("MULTI_HUB_DELAY") is not None:
+        G.set_param(sssp.SSSP_PARAM_MULTI_HUB_DELAY, int(os.environ["MULTI_HUB_DELAY"]))
     out = torch.empty((n, g.V), dtype=torch.int32, device="cuda")
     out2 = torch.empty_like(out)
     for d in deltas:
