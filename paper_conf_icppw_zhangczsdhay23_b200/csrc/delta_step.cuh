@@ -53,7 +53,7 @@ constexpr u32 HUB_CHUNK = 4096;
 #define SSSP_PROBE_L1 1  // dist probes through L1 (a stale value is a safe filter)
 #endif
 #ifndef SSSP_PREFETCH
-#define SSSP_PREFETCH 1  // L2 bulk prefetch of each claimed vertex's arc range
+#define SSSP_PREFETCH 0  // 1: L2 bulk prefetch of each claimed vertex's arc range (session 3: 4 % slower on C4)
 #endif
 #ifndef SSSP_LAT
 #define SSSP_LAT 0  // per-stage latency accounting in the task loop (diagnostics build)
