@@ -594,3 +594,37 @@ def test_distances_async_pipeline(sssp):
         with pytest.raises(sssp.SSSPError) as e:
             G.distances_async(np.empty(g.V, dtype=np.uint32))
         assert e.value.status == sssp.SSSP_ERR_INVALID_ARGUMENT
+
+
+def test_determinism_1000_runs_c1_and_multi(sssp):
+    """SURVEY §4 stress: 1000 repeated runs on a skewed RMAT graph are bit-identical
+    (the fixpoint is unique whatever the asynchronous schedule), and so are 50
+    repeated 32-source multi runs."""
+    import torch
+
+    g = gen.make_config("C1")
+    s = int(gen.sample_sources(g, 1, seed=9)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        dev = torch.empty(g.V, dtype=torch.int32, device="cuda")
+        acc = torch.zeros(g.V, dtype=torch.int64, device="cuda")
+        first = None
+        for k in range(1000):
+            G.run(s, 64)
+            G.distances_async(dev)
+            if first is None:
+                torch.cuda.synchronize()
+                first = dev.clone()
+            acc += (dev != first).to(torch.int64)
+        torch.cuda.synchronize()
+        assert int(acc.sum()) == 0, "runs differ"
+        assert_same(first.cpu().numpy().view(np.uint32), exp, "C1 x1000")
+        srcs = [int(x) for x in gen.sample_sources(g, 32, seed=10)]
+        out = torch.empty((32, g.V), dtype=torch.int32, device="cuda")
+        G.run_multi(srcs, 64, out)
+        ref = out.clone()
+        for _ in range(50):
+            G.run_multi(srcs, 64, out)
+            assert torch.equal(out, ref), "multi runs differ"
+        assert_same(ref[7].cpu().numpy().view(np.uint32), oracle.dijkstra(g.row, g.col, g.w, srcs[7]), "multi lane 7")
