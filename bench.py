@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--sources", type=int, default=64)
     ap.add_argument("--ctas-per-sm", type=int, default=0)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/cpu/e2e)")
+    ap.add_argument("--no-pull", action="store_true", help="push-style phases 2&3 in every bucket")
     ap.add_argument("--multi", action="store_true",
                     help="NEXT-4: a step is one group of up to 32 of the rank's sources through sssp_run_multi")
     return ap.parse_args()
@@ -237,6 +238,9 @@ def main():
     mine = sources[rank::world]
     stream = torch.cuda.Stream(device=dev)
     G = sssp.Graph(g.row, g.col, g.w, device=dev, stream=stream)
+    if gen.CONFIGS[args.config].get("symmetric", True) and not args.no_pull:
+        # the generators symmetrise every config (reading R13): large buckets may pull
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
     if args.ctas_per_sm:
         G.set_param(sssp.SSSP_PARAM_CTAS_PER_SM, args.ctas_per_sm)
     reorder_ms = None
@@ -386,6 +390,7 @@ def main():
         "data": "synthetic",
         "config": {"workload": desc, "V": g.V, "m_edges": g.m, "arcs": g.A, "delta": delta,
                    "reorder": reorder, "reorder_ms": reorder_ms, "sources": len(sources),
+                   "pull_phase2": not args.no_pull,
                    "parallelism": f"replicas x{world} (sources sharded, graph replicated)",
                    "l2": "inputs larger than L2 (arc array %.2f GB > 126 MB L2); dist re-initialised every step" % (8 * g.A / 1e9),
                    "gen_s": round(t_gen, 1), "grid_ctas": st["grid_ctas"], "ring_slots": st["ring_slots"],

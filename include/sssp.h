@@ -212,10 +212,17 @@ typedef enum {
                                       about the same bucket (one SSSP from that vertex per graph
                                       and Delta, which replaces the last sssp_run result); 0 by
                                       plain distance. Results are identical [1] */
-    SSSP_PARAM_MULTI_HUB_DELAY = 10 /* sssp_run_multi on a degree-reordered graph: vertices
+    SSSP_PARAM_MULTI_HUB_DELAY = 10, /* sssp_run_multi on a degree-reordered graph: vertices
                                       of degree > 1024 are queued this many buckets late, so
                                       more of the 32 sources reach a hub before its (long)
                                       adjacency is expanded; 0..16. Results are identical [0] */
+    SSSP_PARAM_PULL_SYMMETRIC = 11 /* 1 = the caller asserts the graph is symmetric (every arc
+                                      (u,v,w) has its reverse (v,u,w), as the generators' graphs
+                                      are, R13): u32 graphs after a weight-sorting sssp_reorder
+                                      then run phases 2&3 of buckets holding >= V/16 entries as a
+                                      pull (each unsettled vertex scans its weight-sorted heavy
+                                      arcs up to the first that cannot win). Same distances;
+                                      wrong distances if the graph is not symmetric [0] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

@@ -48,6 +48,7 @@ SSSP_PARAM_P2_EDGE_BALANCED = 7
 SSSP_PARAM_ADAPTIVE_DELTA = 8
 SSSP_PARAM_MULTI_ALIGN = 9
 SSSP_PARAM_MULTI_HUB_DELAY = 10
+SSSP_PARAM_PULL_SYMMETRIC = 11
 
 INF_U32 = 0xFFFFFFFF
 

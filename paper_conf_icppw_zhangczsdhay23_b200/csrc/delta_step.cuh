@@ -68,6 +68,9 @@ constexpr int UNROLL = SSSP_UNROLL;
 constexpr int IPT = SSSP_IPT;
 constexpr int IPT2 = SSSP_IPT2;
 constexpr int IPT_MAX = IPT > IPT2 ? IPT : IPT2;
+#ifndef SSSP_PULL_DIV
+#define SSSP_PULL_DIV 16u  // pull phase 2 when a bucket holds >= V / 16 entries
+#endif
 #ifndef SSSP_CLAIM_MINPART
 #define SSSP_CLAIM_MINPART 64u  // take a partial batch once this many entries are ready ...
 #endif
@@ -88,7 +91,8 @@ enum : u32 {
   MODE_SWEEP_HEAVY = 6,
   MODE_P2_COMPACT = 7,  // edge-balanced phase 2, step 1: settled entries -> heavy-arc offsets
   MODE_P2_RELAX = 8,    // ... step 2: equal heavy-arc ranges per warp
-  MODE_MERGE = 9        // adaptive Delta: fold the slots (cur, cur_end) into slot cur
+  MODE_MERGE = 9,       // adaptive Delta: fold the slots (cur, cur_end) into slot cur
+  MODE_PULL = 10        // phases 2&3 as a pull over the unsettled vertices (symmetric u32 graphs)
 };
 enum : u32 { ERR_OVERFLOW = 1, ERR_INTERNAL = 2 };
 enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5, SYNC_P2C = 6,
@@ -194,6 +198,7 @@ struct Params {
   // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
   // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL;
   // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries;
+  // bit 7 PULL: pull-style phases 2&3 for large buckets (symmetric u32 graphs, PRO);
   // bits 3/4 adaptive Delta reading A/B (NEXT-1); bit 5 f32 weights (theta level bits)).
   // Params stays <= 128 bytes: larger, it spills around the out-of-line pb_flush call.
   u32 flags;
@@ -915,6 +920,10 @@ __device__ void decide(const Params& p, u32 which) {
     const u32 b = sc[s].p2;
     c->p2_begin = b;
     c->p2_end = tail;
+    if ((p.flags & 128u) && tail - b >= p.V / SSSP_PULL_DIV) {  // large bucket: pull phase 2
+      c->mode = MODE_PULL;
+      return;
+    }
     if ((p.flags & 4u) && tail - b >= (p.flags >> 8)) {  // edge-balanced phase 2
       c->hub_word = 0;
       c->p2_head = 0;
@@ -1435,6 +1444,89 @@ __device__ void p2_relax(const Params& p, Smem& sm) {
   if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
 }
 
+// ------------------------------------------------------ pull phase 2 -----
+// Phases 2&3 of a bucket with many settled vertices, turned around (the
+// direction-optimising idea, valid because the graph is symmetric: v's arc
+// (v, u, w) exists iff u's arc (u, v, w) does). Alg. 2 l.13-17 relaxes the
+// heavy arcs (w >= Delta) of every vertex u settled in bucket cur; here every
+// vertex v not settled yet (dist[v] >= hi) scans its own heavy arcs, which PRO
+// sorted by ascending weight, and takes min(dist[u] + w) over
+// neighbours u whose distance lies in bucket cur. A candidate through bucket
+// cur is >= lo + w, so the scan stops at the first arc with lo + w >= best:
+// most vertices find a hub of the bucket among their lightest heavy arcs and
+// stop early. Every heavy arc out of bucket cur that could improve v is still
+// examined, so the result is the one push-style phase 2 gives.
+template <bool F32, bool PRO>
+__device__ void pull_phase(const Params& p, Smem& sm) {
+  const u32 cur = sm.cur, lim = sm.lim, lane = lane_id();
+  {  // recycle the bucket's queue entries (push-style phase 2 consumes them)
+    u64* q = p.items + (u64)(cur & p.kmask) * p.cap;
+    for (i64 i = sm.p2_begin + (i64)blockIdx.x * blockDim.x + threadIdx.x; i < sm.p2_end;
+         i += (i64)gridDim.x * blockDim.x)
+      st_relaxed_u64(q + i, SENTINEL);
+  }
+  const u64 lo = (u64)cur * p.delta_u, hi = lo + p.delta_u;
+  u32 c_pull = 0, c_arcs = 0;
+  const u64 pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
+  const i64 nt = (i64)gridDim.x * blockDim.x;
+  for (i64 b = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL; b < p.V; b += nt) {
+    const i64 v = b + lane;
+    u32 dv = 0, j = 0, e = 0;
+    bool act = v < p.V;
+    if (act) {
+      dv = ld_cg(p.dist + v);
+      act = (u64)dv >= hi;
+    }
+    if (act) {
+      const uint2 r = p.rowc[v];
+      j = PRO ? r.y : r.x;
+      e = p.rowc[v + 1].x;
+      act = j < e;
+    }
+    u32 best = dv;
+    while (__any_sync(SSSP_FULL_MASK, act)) {
+      uint2 a[UNROLL];
+      u32 du[UNROLL];
+      bool ok[UNROLL];
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) a[k] = ld_arc(p.arcs + j + k, act && j + k < e, pol_stream);
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        ok[k] = act && j + k < e && lo + a[k].y < (u64)best;  // ascending w: later arcs cannot win
+        if (!PRO) ok[k] = ok[k] && a[k].y >= p.delta_bits;  // heavy arcs only
+        du[k] = ld_probe(p.dist + a[k].x, ok[k], pol_keep);
+      }
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        if (ok[k] && (u64)du[k] >= lo && (u64)du[k] < hi) {  // u settled in bucket cur
+          const u64 cand = (u64)du[k] + a[k].y;
+          if (cand < (u64)best) best = (u32)min(cand, (u64)NONE);
+        }
+      }
+      if (act) c_arcs += min((u32)UNROLL, e - j);
+      j += UNROLL;
+      act = act && j < e && (PRO ? ok[UNROLL - 1] : true);
+    }
+    bool want[UNROLL] = {};
+    u32 vv[UNROLL] = {}, nd[UNROLL] = {};
+    if (v < p.V && best < dv) {
+      if (best >= NONE) {
+        atomicOr(&p.ctl->err, ERR_OVERFLOW);
+      } else {
+        atomicMin(p.dist + v, best);
+        want[0] = true;
+        vv[0] = (u32)v;
+        nd[0] = best;
+        ++c_pull;
+      }
+    }
+    stage_pushes<F32>(p, sm, lim, NONE, want, vv, nd);
+  }
+  if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
+  st_add(sm, ST_HEAVY, c_arcs);
+  st_add(sm, ST_HEAVYV, c_pull);
+}
+
 // Rescan stage 1: clear every queue entry still holding a value.
 __device__ void rescan_clear(const Params& p) {
   const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
@@ -1575,6 +1667,9 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
       grid_barrier(p, sm, SYNC_P1);
     } else if (mode == MODE_PHASE2) {
       phase2<F32, PRO, ABL>(p, sm);
+      grid_barrier(p, sm, SYNC_P2);
+    } else if (!F32 && mode == MODE_PULL) {  // u32 graphs only
+      if constexpr (!F32) pull_phase<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (ABL && mode == MODE_MERGE) {  // extended build only (adaptive Delta)
       if constexpr (ABL) merge_slots<F32>(p, sm);

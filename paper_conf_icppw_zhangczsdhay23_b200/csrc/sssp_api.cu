@@ -97,7 +97,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0;
   i64 hub_ids_cached = -1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
@@ -331,6 +331,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_MULTI_HUB_DELAY:
       if (v < 0 || v > 16) return fail(SSSP_ERR_INVALID_ARGUMENT, "hub delay in [0,16]");
       g->p_hub_delay = v;
+      return SSSP_OK;
+    case SSSP_PARAM_PULL_SYMMETRIC:
+      if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "pull is 0 or 1");
+      g->p_pull = v;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
@@ -684,6 +688,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
   if (adapt) p.flags |= (dp.ai.mode == 2 ? 16u : 8u) | (pro ? 64u : 0u);
   if (f32) p.flags |= 32u;
+  if (g->p_pull && pro && !f32 && !adapt) p.flags |= 128u;  // caller asserted a symmetric graph
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal, dp.ai);

@@ -47,6 +47,7 @@ def test_config_parity(sssp, name, n_exact, n_cert):
     srcs = gen.sample_sources(g, n_exact + n_cert, seed=7)
     with sssp.Graph(g.row, g.col, g.w) as G:
         G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)  # as bench.py (symmetric generator graphs)
         for i, s in enumerate(srcs):
             got = G.sssp(int(s), delta).copy()
             st = G.stats()
@@ -175,6 +176,7 @@ def test_c5_full_size_certificates(sssp):
     srcs = [int(s) for s in gen.sample_sources(g, 32, seed=7)]
     with sssp.Graph(g.row, g.col, g.w) as G:
         G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)  # as bench.py
         d = G.sssp(srcs[0], gen.CONFIGS["C5"]["delta"]).copy()
         assert oracle.certificate(g.row, g.col, g.w, srcs[0], d) == -1, "C5 single-source certificate"
         out = torch.empty((32, g.V), dtype=torch.int32, device="cuda")

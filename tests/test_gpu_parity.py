@@ -628,3 +628,27 @@ def test_determinism_1000_runs_c1_and_multi(sssp):
             G.run_multi(srcs, 64, out)
             assert torch.equal(out, ref), "multi runs differ"
         assert_same(ref[7].cpu().numpy().view(np.uint32), oracle.dijkstra(g.row, g.col, g.w, srcs[7]), "multi lane 7")
+
+
+@pytest.mark.parametrize("scale,deltas", [(12, (1, 4, 16, 64, 200)), (14, (8, 16, 32))])
+@pytest.mark.parametrize("flags", [3, 2])
+def test_pull_phase2_parity(sssp, scale, deltas, flags):
+    """SSSP_PARAM_PULL_SYMMETRIC: large buckets run phases 2&3 as a pull over the
+    unsettled vertices (symmetric generator graphs); distances unchanged."""
+    g = gen.kronecker(scale, 16, seed=60 + scale)
+    srcs = gen.sample_sources(g, 3, seed=5)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder(flags)
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        for s in srcs:
+            exp = oracle.dijkstra(g.row, g.col, g.w, int(s))
+            for d in deltas:
+                assert_same(G.sssp(int(s), d), exp, f"pull s{scale} flags={flags} delta={d} src={s}")
+    gg = gen.grid(300, 200, p=0.2, seed=5)
+    s = int(gen.sample_sources(gg, 1, seed=1)[0])
+    exp = oracle.dijkstra(gg.row, gg.col, gg.w, s)
+    with sssp.Graph(gg.row, gg.col, gg.w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        for d in (50, 1600, 100000):
+            assert_same(G.sssp(s, d), exp, f"pull grid delta={d}")
