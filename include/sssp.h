@@ -218,7 +218,7 @@ typedef enum {
                                       adjacency is expanded; 0..16. Results are identical [0] */
     SSSP_PARAM_PULL_SYMMETRIC = 11 /* 1 = the caller asserts the graph is symmetric (every arc
                                       (u,v,w) has its reverse (v,u,w), as the generators' graphs
-                                      are, R13): u32 graphs after a weight-sorting sssp_reorder
+                                      are, R13): graphs after a weight-sorting sssp_reorder
                                       then run phases 2&3 of buckets holding >= V/16 entries as a
                                       pull (each unsettled vertex scans its weight-sorted heavy
                                       arcs up to the first that cannot win). Same distances;

@@ -198,7 +198,8 @@ struct Params {
   // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
   // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL;
   // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries;
-  // bit 7 PULL: pull-style phases 2&3 for large buckets (symmetric u32 graphs, PRO);
+  // bit 7 PULL: pull-style phases 2&3 for large buckets (symmetric graphs, PRO; f32 graphs
+  // then carry Delta's bits in delta_u);
   // bits 3/4 adaptive Delta reading A/B (NEXT-1); bit 5 f32 weights (theta level bits)).
   // Params stays <= 128 bytes: larger, it spills around the out-of-line pb_flush call.
   u32 flags;
@@ -1465,7 +1466,11 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
          i += (i64)gridDim.x * blockDim.x)
       st_relaxed_u64(q + i, SENTINEL);
   }
-  const u64 lo = (u64)cur * p.delta_u, hi = lo + p.delta_u;
+  // u32: bucket cur = [lo, hi). f32 (delta_u holds Delta's bits): membership by bucket_of, and
+  // lo_f <= every distance of bucket cur (cur * Delta rounded down, less 2^-20 relative), so
+  // fl(lo_f + w) is a lower bound of fl(du + w) for every u of the bucket (fl is monotone).
+  const u64 lo = F32 ? 0 : (u64)cur * p.delta_u, hi = F32 ? 0 : lo + p.delta_u;
+  const float lo_f = (F32 && cur) ? __fmul_rd(__fmul_rd((float)cur, __uint_as_float(p.delta_u)), 0.99999905f) : 0.f;
   u32 c_pull = 0, c_arcs = 0;
   const u64 pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
   const i64 nt = (i64)gridDim.x * blockDim.x;
@@ -1475,7 +1480,7 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
     bool act = v < p.V;
     if (act) {
       dv = ld_cg(p.dist + v);
-      act = (u64)dv >= hi;
+      act = F32 ? bucket_of<true>(p, dv) > cur : (u64)dv >= hi;
     }
     if (act) {
       const uint2 r = p.rowc[v];
@@ -1492,15 +1497,23 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
       for (int k = 0; k < UNROLL; ++k) a[k] = ld_arc(p.arcs + j + k, act && j + k < e, pol_stream);
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
-        ok[k] = act && j + k < e && lo + a[k].y < (u64)best;  // ascending w: later arcs cannot win
+        ok[k] = act && j + k < e &&  // ascending w: once the bound fails, later arcs cannot win
+                (F32 ? __float_as_uint(__fadd_rn(lo_f, __uint_as_float(a[k].y))) < best : lo + a[k].y < (u64)best);
         if (!PRO) ok[k] = ok[k] && a[k].y >= p.delta_bits;  // heavy arcs only
         du[k] = ld_probe(p.dist + a[k].x, ok[k], pol_keep);
       }
 #pragma unroll
       for (int k = 0; k < UNROLL; ++k) {
-        if (ok[k] && (u64)du[k] >= lo && (u64)du[k] < hi) {  // u settled in bucket cur
-          const u64 cand = (u64)du[k] + a[k].y;
-          if (cand < (u64)best) best = (u32)min(cand, (u64)NONE);
+        if constexpr (F32) {
+          if (ok[k] && bucket_of<true>(p, du[k]) == cur) {  // u settled in bucket cur
+            const u32 cand = __float_as_uint(__fadd_rn(__uint_as_float(du[k]), __uint_as_float(a[k].y)));
+            best = min(best, cand);
+          }
+        } else {
+          if (ok[k] && (u64)du[k] >= lo && (u64)du[k] < hi) {  // u settled in bucket cur
+            const u64 cand = (u64)du[k] + a[k].y;
+            if (cand < (u64)best) best = (u32)min(cand, (u64)NONE);
+          }
         }
       }
       if (act) c_arcs += min((u32)UNROLL, e - j);
@@ -1510,7 +1523,7 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
     bool want[UNROLL] = {};
     u32 vv[UNROLL] = {}, nd[UNROLL] = {};
     if (v < p.V && best < dv) {
-      if (best >= NONE) {
+      if (!F32 && best >= NONE) {
         atomicOr(&p.ctl->err, ERR_OVERFLOW);
       } else {
         atomicMin(p.dist + v, best);
@@ -1668,8 +1681,8 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     } else if (mode == MODE_PHASE2) {
       phase2<F32, PRO, ABL>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
-    } else if (!F32 && mode == MODE_PULL) {  // u32 graphs only
-      if constexpr (!F32) pull_phase<F32, PRO>(p, sm);
+    } else if (mode == MODE_PULL) {
+      pull_phase<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (ABL && mode == MODE_MERGE) {  // extended build only (adaptive Delta)
       if constexpr (ABL) merge_slots<F32>(p, sm);

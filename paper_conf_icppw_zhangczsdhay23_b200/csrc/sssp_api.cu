@@ -688,7 +688,10 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
   if (adapt) p.flags |= (dp.ai.mode == 2 ? 16u : 8u) | (pro ? 64u : 0u);
   if (f32) p.flags |= 32u;
-  if (g->p_pull && pro && !f32 && !adapt) p.flags |= 128u;  // caller asserted a symmetric graph
+  if (g->p_pull && pro && !adapt && (f32 ? dp.inv != 0.f : dp.delta_u != 0xFFFFFFFFu)) {  // caller asserted symmetry
+    p.flags |= 128u;
+    if (f32) p.delta_u = dp.delta_bits;  // pull_phase needs Delta itself (bucket_of uses inv_delta)
+  }
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal, dp.ai);

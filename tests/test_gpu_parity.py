@@ -652,3 +652,18 @@ def test_pull_phase2_parity(sssp, scale, deltas, flags):
         G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
         for d in (50, 1600, 100000):
             assert_same(G.sssp(s, d), exp, f"pull grid delta={d}")
+
+
+@pytest.mark.parametrize("deltas", [(0.01, 0.05, 0.1, 0.3, float("inf"))])
+def test_pull_phase2_parity_f32(sssp, deltas):
+    """The f32 pull: membership by bucket_of, the early stop by the lower bound
+    fl(lo_f + w) (lo_f <= every distance of the bucket); bit-exact."""
+    g = gen.kronecker(13, 16, seed=71, weights="f32")
+    srcs = gen.sample_sources(g, 3, seed=6)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        for s in srcs:
+            exp = oracle.dijkstra(g.row, g.col, g.w, int(s))
+            for d in deltas:
+                assert_same(G.sssp(int(s), d), exp, f"pull f32 delta={d} src={s}")
