@@ -18,6 +18,7 @@ def main():
     ap.add_argument("--runs", type=int, default=8)
     ap.add_argument("--rounds", type=int, default=3)
     ap.add_argument("--deltas", type=float, nargs="*", default=None)
+    ap.add_argument("--param", action="append", default=[], help="PARAM_ID=VALUE (sssp_set_param)")
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     import torch  # noqa: F401  (CUDA context)
@@ -39,6 +40,10 @@ def main():
         assert L.sssp_graph_create(ctypes.byref(h), 0, g.V, g.A, g.row.ctypes.data, g.col.ctypes.data,
                                    g.w.ctypes.data, wt, 0, None) == 0
         assert L.sssp_reorder(h) == 0
+        L.sssp_set_param.argtypes = [P, I, I64]
+        for kv in a.param:
+            k, v = kv.split("=")
+            assert L.sssp_set_param(h, int(k), int(v)) == 0
         assert L.sssp_run(h, int(srcs[0]), float(delta)) == 0
         t, n = ctypes.c_double(), ctypes.c_int64()
         L.sssp_kernel_time(h, ctypes.byref(t), ctypes.byref(n), 1)
