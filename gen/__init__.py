@@ -177,7 +177,7 @@ def scramble(x, scale, seed):
 # the paper's 0.1, flat within 0.1-0.15.
 CONFIGS = {
     "C1": dict(kind="kron", scale=16, edgefactor=16, seed=1, weights="u32", delta=64),
-    "C2": dict(kind="grid", W=4894, H=4894, p=0.2, seed=2, weights="u32", delta=1600),
+    "C2": dict(kind="grid", W=4894, H=4894, p=0.2, seed=2, weights="u32", delta=6400),
     "C3": dict(kind="kron", scale=22, edgefactor=16, seed=3, weights="f32", delta=0.1),
     "C4": dict(kind="kron", scale=24, edgefactor=16, seed=4, weights="u32", delta=16),
     "C5": dict(kind="kron", scale=26, edgefactor=16, seed=5, weights="u32", delta=16),

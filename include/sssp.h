@@ -186,7 +186,7 @@ typedef enum {
     SSSP_PARAM_RING_SLOTS = 0,     /* K bucket queues, power of two in [4,64]; 0 = auto [0] */
     SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
     SSSP_PARAM_SLOT_CAPACITY = 2,  /* entries per bucket queue; 0 = auto (2.5 V + 64Ki) [0] */
-    SSSP_PARAM_CLAIM_MAX = 3,      /* max queue entries one CTA claims at once (1..1024) [1024] */
+    SSSP_PARAM_CLAIM_MAX = 3,      /* max queue entries one CTA claims at once (1..512) [512] */
     SSSP_PARAM_L2_PERSIST = 4,     /* 1: keep dist[] in a persisting L2 window (raises the
                                       device's persisting-L2 limit; never lowers it) [1] */
     SSSP_PARAM_ADWL = 5,           /* ablation: 1 adaptive thread/warp/CTA bins + hub chunks
@@ -216,13 +216,24 @@ typedef enum {
                                       of degree > 1024 are queued this many buckets late, so
                                       more of the 32 sources reach a hub before its (long)
                                       adjacency is expanded; 0..16. Results are identical [0] */
-    SSSP_PARAM_PULL_SYMMETRIC = 11 /* 1 = the caller asserts the graph is symmetric (every arc
+    SSSP_PARAM_PULL_SYMMETRIC = 11, /* 1 = the caller asserts the graph is symmetric (every arc
                                       (u,v,w) has its reverse (v,u,w), as the generators' graphs
                                       are, R13): graphs after a weight-sorting sssp_reorder
                                       then run phases 2&3 of buckets holding >= V/16 entries as a
                                       pull (each unsettled vertex scans its weight-sorted heavy
                                       arcs up to the first that cannot win). Same distances;
                                       wrong distances if the graph is not symmetric [0] */
+    SSSP_PARAM_LOCAL_CHASE = 12    /* 2: when no arc is heavy at the run's Delta (max weight <
+                                      Delta, fixed Delta), a phase-1 push into
+                                      the current bucket stays in the pushing CTA's shared
+                                      memory (up to one batch) and that CTA relaxes it next,
+                                      skipping the global queue round trip; the bucket's
+                                      pending count stays > 0 until the CTA's chain is done
+                                      (P:1063-1065 leaves the near-list layout open, R10).
+                                      1 = the same, only on sparse graphs (A <= 8 V, e.g. road
+                                      networks: thin frontiers; on dense ones the CTA-local
+                                      depth-first order re-relaxes more). Same distances;
+                                      0 = always through the global queue [1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

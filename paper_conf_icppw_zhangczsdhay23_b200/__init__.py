@@ -49,6 +49,7 @@ SSSP_PARAM_ADAPTIVE_DELTA = 8
 SSSP_PARAM_MULTI_ALIGN = 9
 SSSP_PARAM_MULTI_HUB_DELAY = 10
 SSSP_PARAM_PULL_SYMMETRIC = 11
+SSSP_PARAM_LOCAL_CHASE = 12
 
 INF_U32 = 0xFFFFFFFF
 

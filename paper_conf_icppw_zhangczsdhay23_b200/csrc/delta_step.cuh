@@ -215,6 +215,8 @@ constexpr u32 SB_CAP = 32 * IPT_MAX;           // thread-bin entries per warp
 #define SSSP_PB_CAP 256u
 #endif
 constexpr u32 PB_CAP = SSSP_PB_CAP;  // staged pushes per warp (>= 32 * UNROLL)
+constexpr u32 LOC_CAP = BATCH;       // CTA-local chase list: one phase-1 batch
+constexpr u32 LOCAL_CHASE = 1u << 16;  // Params::claim_max bit (claim_max itself <= BATCH)
 
 struct Smem {
   // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
@@ -239,6 +241,10 @@ struct Smem {
   u32 pb_n[DS_WARPS];
   unsigned long long st[ST_N];
   u32 claim_h, claim_n, claim_src;
+  // CTA-local chase (LOCAL_CHASE): phase-1 pushes into the current bucket kept in shared
+  // memory and processed by this CTA next, without the global queue round trip
+  u64 loc[LOC_CAP];
+  u32 loc_n, loc_on;
   // control snapshot
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
   u32 cur_end, rowc_off, theta_bits;  // bucket end (fine slots), light/heavy level
@@ -367,6 +373,21 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
       ok = false;
+    }
+    // CTA-local chase: this CTA relaxes the vertex itself in its next batch. Only enabled
+    // when no arc is heavy at this Delta (phase 2 then needs no settled list in the queue).
+    const bool lc = ok && in_cur && sm.loc_on;
+    const u32 lm = __ballot_sync(SSSP_FULL_MASK, lc);
+    if (lm) {
+      const u32 ld = __ffs(lm) - 1;
+      u32 base = 0;
+      if (lane == ld) base = atomicAdd(&sm.loc_n, (u32)__popc(lm));
+      base = __shfl_sync(SSSP_FULL_MASK, base, ld);
+      const u32 li = base + __popc(lm & lanemask_lt());
+      if (lc && li < LOC_CAP) {
+        sm.loc[li] = e;
+        ok = false;
+      }
     }
     if (ok && x > lim) {  // beyond the ring horizon: rescan later
       atomicMin(&p.ctl->far_min, x);
@@ -1091,23 +1112,34 @@ __device__ void phase1(const Params& p, Smem& sm) {
   SlotCtl* sc = p.sc + slot;
   u64* q = p.items + (u64)slot * p.cap;
   const u32 G = gridDim.x;
+  const u32 claim_max = p.claim_max & (LOCAL_CHASE - 1);
   u32 my_next = 0, my_end = 0;  // thread 0: claimed ticket range
+  u32 owed = 0;  // thread 0: completions of claimed entries held back while the CTA chases locally
+  if (threadIdx.x == 0) sm.loc_on = (!ABL && (p.claim_max & LOCAL_CHASE)) ? 1u : 0u;
   for (;;) {
     if (threadIdx.x == 0) {
       const long long t_c = clock64();
-      u32 n = 0, h = 0, ns = 32, waited = 0;
-      if (ABL && (p.flags & 2u)) {  // level-synchronous: only this level's entries, all already written
+      u32 n = 0, h = 0, ns = 32, waited = 0, loc = 0;
+      if (sm.loc_n) {  // the CTA's own pushes first: pend stays > 0 (owed) until they are done
+        n = min(sm.loc_n, LOC_CAP);
+        loc = 1;
+      } else if (owed) {
+        atomicAdd(&sc->word, (u64)0 - (u64)owed);  // completion of the chased-from entries
+        owed = 0;
+      }
+      if (loc) {
+      } else if (ABL && (p.flags & 2u)) {  // level-synchronous: only this level's entries, all already written
         const u32 re = sm.round_end;
-        const u32 c = min(max(re / (2 * G), 8u), min(p.claim_max, BATCH));
+        const u32 c = min(max(re / (2 * G), 8u), min(claim_max, BATCH));
         h = ld_relaxed_u32(&sc->head) < re ? atomicAdd(&sc->head, c) : re;
         n = h < re ? min(c, re - h) : 0u;
       }
-      for (; !(ABL && (p.flags & 2u));) {
+      for (; !loc && !(ABL && (p.flags & 2u));) {
         const u64 wv = ld_relaxed_u64(&sc->word);
         const u32 tail = min((u32)(wv >> 32), p.cap);
         if (my_next >= my_end && my_end < p.cap) {
           // claim size grows with the queue: small early (spread work), up to claim_max
-          u32 c = min(max(tail / (2 * G), 8u), p.claim_max);
+          u32 c = min(max(tail / (2 * G), 8u), claim_max);
           my_next = atomicAdd(&sc->head, c);
           my_end = my_next + c;
         }
@@ -1131,19 +1163,26 @@ __device__ void phase1(const Params& p, Smem& sm) {
       }
       sm.claim_n = n;
       sm.claim_h = h;
+      sm.claim_src = loc;
       sm.st[ST_P_CLAIM] += (unsigned long long)(clock64() - t_c);
     }
     __syncthreads();
     const u32 n = sm.claim_n;
     if (n == 0) break;
     const u32 h = sm.claim_h;
+    const bool loc = sm.claim_src != 0;
     u64 it[IPT];
     bool has[IPT];
 #pragma unroll
     for (int i = 0; i < IPT; ++i) {
       const u32 my = batch_item_index(i);
       has[i] = my < n;
-      it[i] = has[i] ? ld_relaxed_u64(q + h + my) : SENTINEL;
+      it[i] = has[i] ? (loc ? sm.loc[my] : ld_relaxed_u64(q + h + my)) : SENTINEL;
+    }
+    if (loc) {  // list taken: empty it before this batch pushes again
+      __syncthreads();
+      if (threadIdx.x == 0) sm.loc_n = 0;
+      __syncthreads();
     }
 #pragma unroll
     for (int i = 0; i < IPT; ++i) {
@@ -1158,8 +1197,14 @@ __device__ void phase1(const Params& p, Smem& sm) {
       process_batch<F32, PRO, 1, IPT, true, ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
     else
       process_batch<F32, PRO, 1, IPT, !ABL, ABL>(p, sm, it, has, lim, SRC_QUEUE, slot);
-    if (threadIdx.x == 0) atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
+    if (threadIdx.x == 0 && !loc) {
+      if (sm.loc_on)
+        owed += n;  // completion deferred until the local list is drained
+      else
+        atomicAdd(&sc->word, (u64)0 - (u64)n);  // completion
+    }
   }
+  if (threadIdx.x == 0) sm.loc_on = 0;
 }
 
 template <bool F32, bool PRO, bool ABL>
@@ -1661,6 +1706,8 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
   if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
   if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
+    sm.loc_n = 0;
+    sm.loc_on = 0;
     volatile Ctl* vc = p.ctl;
     sm.mode = vc->mode;
     sm.cur = vc->cur;

@@ -667,3 +667,33 @@ def test_pull_phase2_parity_f32(sssp, deltas):
             exp = oracle.dijkstra(g.row, g.col, g.w, int(s))
             for d in deltas:
                 assert_same(G.sssp(int(s), d), exp, f"pull f32 delta={d} src={s}")
+
+
+@pytest.mark.gpu
+def test_local_chase_parity(sssp):
+    """SSSP_PARAM_LOCAL_CHASE (2 forced, 1 auto on sparse graphs, while max w < Delta):
+    in-bucket phase-1 pushes stay in the pushing CTA's shared memory. Distances
+    bit-exact with it on and off: grids (hundreds of buckets), Kronecker hubs that
+    overflow the one-batch local list (Delta = inf: one bucket, Bellman-Ford mode),
+    f32 weights, unreordered graphs; valid updates = reachable - 1 either way."""
+    cases = [(gen.grid(300, 200, p=0.2, seed=5), (101, 400, 1600, float("inf")), (True, False)),
+             (gen.kronecker(14, 16, seed=71), (101, 300, float("inf")), (True, False)),
+             (gen.kronecker(13, 16, seed=72, weights="f32"), (1.5, 4.0, float("inf")), (True,))]
+    for g, deltas, reorders in cases:
+        srcs = gen.sample_sources(g, 2, seed=3)
+        exp = {int(s): oracle.dijkstra(g.row, g.col, g.w, int(s)) for s in srcs}
+        for reorder in reorders:
+            with sssp.Graph(g.row, g.col, g.w) as G:
+                if reorder:
+                    G.reorder()
+                for local in (2, 1, 0):
+                    G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, local)
+                    for d in deltas:
+                        for s in srcs:
+                            e = exp[int(s)]
+                            what = f"local={local} reorder={reorder} {g.wtype} V={g.V} delta={d} src={s}"
+                            assert_same(G.sssp(int(s), d), e, what)
+                            st = G.stats()
+                            reach = int(np.count_nonzero(e != (INF if g.wtype == "u32" else np.float32(np.inf))))
+                            assert st["reachable"] == reach, what
+                            assert st["updates"] >= reach - 1, what
