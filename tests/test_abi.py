@@ -87,3 +87,16 @@ def test_no_oracle_in_product_path():
                 assert "import oracle" not in txt and "from oracle" not in txt and "oracle.h" not in txt, f
     out = subprocess.check_output(["nm", "-D", os.path.join(pkg, "libsssp.so")]).decode()
     assert "oracle_" not in out
+
+
+def test_binding_constants_match_header(lib):
+    """Every SSSP_* enumerator of include/sssp.h has the same value in the binding."""
+    txt = re.sub(r"/\*.*?\*/", "", open(HDR).read(), flags=re.S)
+    consts = {k: int(v) for k, v in re.findall(r"\b(SSSP_[A-Z0-9_]+)\s*=\s*(\d+)", txt)}
+    assert "SSSP_PARAM_LOCAL_CHASE" in consts
+    for k, v in consts.items():
+        if k.startswith("SSSP_PARAM_"):
+            assert getattr(lib, k) == v, k
+    for k, v in consts.items():
+        if hasattr(lib, k):
+            assert getattr(lib, k) == v, k
