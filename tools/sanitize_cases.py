@@ -45,6 +45,18 @@ def main():
                 G.wait()
                 same(pin.numpy(), exp, f"{wt} async")
         print(f"sanitize cases {wt}: OK", flush=True)
+    # CTA-local chase (SSSP_PARAM_LOCAL_CHASE): a grid in auto mode, a Kronecker graph forced
+    # (hubs overflow the one-batch local list), Delta above the max weight so no arc is heavy
+    for g, d in ((gen.grid(60, 40, p=0.2, seed=3), 400), (gen.kronecker(10, 16, seed=5), 101)):
+        s = int(gen.sample_sources(g, 1, seed=2)[0])
+        exp = oracle.dijkstra(g.row, g.col, g.w, s)
+        with sssp.Graph(g.row, g.col, g.w) as G:
+            G.set_param(sssp.SSSP_PARAM_CTAS_PER_SM, 1)
+            G.reorder()
+            for local in (1, 2):
+                G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, local)
+                same(G.sssp(s, d), exp, f"local chase {local} V={g.V}")
+    print("sanitize cases local chase: OK", flush=True)
 
 
 if __name__ == "__main__":
