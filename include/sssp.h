@@ -223,7 +223,7 @@ typedef enum {
                                       pull (each unsettled vertex scans its weight-sorted heavy
                                       arcs up to the first that cannot win). Same distances;
                                       wrong distances if the graph is not symmetric [0] */
-    SSSP_PARAM_LOCAL_CHASE = 12    /* 2: when no arc is heavy at the run's Delta (max weight <
+    SSSP_PARAM_LOCAL_CHASE = 12,   /* 2: when no arc is heavy at the run's Delta (max weight <
                                       Delta, fixed Delta), a phase-1 push into
                                       the current bucket stays in the pushing CTA's shared
                                       memory (up to one batch) and that CTA relaxes it next,
@@ -234,6 +234,8 @@ typedef enum {
                                       networks: thin frontiers; on dense ones the CTA-local
                                       depth-first order re-relaxes more). Same distances;
                                       0 = always through the global queue [1] */
+    SSSP_PARAM_LOCAL_LIMIT = 13    /* local-chase entries a CTA keeps (1..512); pushes beyond
+                                      go to the global queue, where idle CTAs can take them [512] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

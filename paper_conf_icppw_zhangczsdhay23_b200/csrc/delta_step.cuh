@@ -216,7 +216,8 @@ constexpr u32 SB_CAP = 32 * IPT_MAX;           // thread-bin entries per warp
 #endif
 constexpr u32 PB_CAP = SSSP_PB_CAP;  // staged pushes per warp (>= 32 * UNROLL)
 constexpr u32 LOC_CAP = BATCH;       // CTA-local chase list: one phase-1 batch
-constexpr u32 LOCAL_CHASE = 1u << 16;  // Params::claim_max bit (claim_max itself <= BATCH)
+constexpr u32 LOCAL_CHASE = 1u << 16;  // Params::claim_max bit (claim_max itself <= BATCH) ...
+constexpr u32 LOCAL_LIM_SHIFT = 20;     // ... and bits 20-29: entries kept locally (<= LOC_CAP)
 
 struct Smem {
   // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
@@ -244,7 +245,7 @@ struct Smem {
   // CTA-local chase (LOCAL_CHASE): phase-1 pushes into the current bucket kept in shared
   // memory and processed by this CTA next, without the global queue round trip
   u64 loc[LOC_CAP];
-  u32 loc_n, loc_on;
+  u32 loc_n, loc_on, loc_lim;
   // control snapshot
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
   u32 cur_end, rowc_off, theta_bits;  // bucket end (fine slots), light/heavy level
@@ -384,7 +385,7 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
       if (lane == ld) base = atomicAdd(&sm.loc_n, (u32)__popc(lm));
       base = __shfl_sync(SSSP_FULL_MASK, base, ld);
       const u32 li = base + __popc(lm & lanemask_lt());
-      if (lc && li < LOC_CAP) {
+      if (lc && li < sm.loc_lim) {  // the rest goes to the global queue, where idle CTAs find it
         sm.loc[li] = e;
         ok = false;
       }
@@ -1112,16 +1113,19 @@ __device__ void phase1(const Params& p, Smem& sm) {
   SlotCtl* sc = p.sc + slot;
   u64* q = p.items + (u64)slot * p.cap;
   const u32 G = gridDim.x;
-  const u32 claim_max = p.claim_max & (LOCAL_CHASE - 1);
+  const u32 claim_max = p.claim_max & (LOCAL_CHASE - 1);  // claim_max <= BATCH
   u32 my_next = 0, my_end = 0;  // thread 0: claimed ticket range
   u32 owed = 0;  // thread 0: completions of claimed entries held back while the CTA chases locally
-  if (threadIdx.x == 0) sm.loc_on = (!ABL && (p.claim_max & LOCAL_CHASE)) ? 1u : 0u;
+  if (threadIdx.x == 0) {
+    sm.loc_on = (!ABL && (p.claim_max & LOCAL_CHASE)) ? 1u : 0u;
+    sm.loc_lim = min((p.claim_max >> LOCAL_LIM_SHIFT) & 1023u, LOC_CAP);
+  }
   for (;;) {
     if (threadIdx.x == 0) {
       const long long t_c = clock64();
       u32 n = 0, h = 0, ns = 32, waited = 0, loc = 0;
       if (sm.loc_n) {  // the CTA's own pushes first: pend stays > 0 (owed) until they are done
-        n = min(sm.loc_n, LOC_CAP);
+        n = min(sm.loc_n, sm.loc_lim);
         loc = 1;
       } else if (owed) {
         atomicAdd(&sc->word, (u64)0 - (u64)owed);  // completion of the chased-from entries

@@ -97,7 +97,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP;
   i64 hub_ids_cached = -1;
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
@@ -339,6 +339,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_LOCAL_CHASE:
       if (v < 0 || v > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "local chase is 0, 1 or 2");
       g->p_local = v;
+      return SSSP_OK;
+    case SSSP_PARAM_LOCAL_LIMIT:
+      if (v < 1 || v > (i64)LOC_CAP) return fail(SSSP_ERR_INVALID_ARGUMENT, "local limit in [1,%u]", LOC_CAP);
+      g->p_local_lim = v;
       return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
@@ -690,7 +694,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   // (1) also asks for a sparse graph (A <= 8 V: thin, long frontiers as on road networks),
   // where the chase cuts per-hop latency; on dense graphs it measured slower (C1 2x)
   if (g->p_local && !adapt && !g->p_sync && g->maxw_bits < dp.delta_bits && (g->p_local == 2 || g->A <= 8 * g->V))
-    p.claim_max |= LOCAL_CHASE;
+    p.claim_max |= LOCAL_CHASE | ((u32)g->p_local_lim << LOCAL_LIM_SHIFT);
   p.p2o = g->p2o;
   p.flags = (g->p_adwl ? 1u : 0u) | (g->p_sync ? 2u : 0u);
   // edge-balanced phase 2 (not in the static thread-per-vertex ablation)

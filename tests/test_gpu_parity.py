@@ -686,12 +686,13 @@ def test_local_chase_parity(sssp):
             with sssp.Graph(g.row, g.col, g.w) as G:
                 if reorder:
                     G.reorder()
-                for local in (2, 1, 0):
+                for local, lim in ((2, 512), (2, 8), (1, 64), (0, 512)):
                     G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, local)
+                    G.set_param(sssp.SSSP_PARAM_LOCAL_LIMIT, lim)
                     for d in deltas:
                         for s in srcs:
                             e = exp[int(s)]
-                            what = f"local={local} reorder={reorder} {g.wtype} V={g.V} delta={d} src={s}"
+                            what = f"local={local} lim={lim} reorder={reorder} {g.wtype} V={g.V} delta={d} src={s}"
                             assert_same(G.sssp(int(s), d), e, what)
                             st = G.stats()
                             reach = int(np.count_nonzero(e != (INF if g.wtype == "u32" else np.float32(np.inf))))
