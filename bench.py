@@ -235,7 +235,9 @@ def main():
     g = gen.make_config(args.config)
     t_gen = time.perf_counter() - t_gen
     sources = gen.sample_sources(g, args.sources, seed=7)
-    mine = sources[rank::world]
+    from paper_conf_icppw_zhangczsdhay23_b200 import batch
+
+    mine = batch.shard_sources(sources, rank, world)  # contiguous blocks (batch.py)
     stream = torch.cuda.Stream(device=dev)
     G = sssp.Graph(g.row, g.col, g.w, device=dev, stream=stream)
     if gen.CONFIGS[args.config].get("symmetric", True) and not args.no_pull:
@@ -293,8 +295,6 @@ def main():
     # the N distance rows are gathered to rank 0 over NCCL and copied to pinned host
     e2e_multi = None
     if world > 1 and not args.no_e2e and not args.profile:
-        from paper_conf_icppw_zhangczsdhay23_b200 import batch
-
         ne = min(args.steps, 16)
         # rank 0 copies step k's gathered rows to pinned host memory on a copy stream while
         # step k+1 runs (double-buffered); every copy finishes inside the timed region
@@ -306,7 +306,7 @@ def main():
         t0 = time.perf_counter()
         for k in range(ne):
             step_src = sources[(k * world) % len(sources):][:world]
-            rows = batch.run_sharded(G, step_src, delta, dst=0)
+            rows = batch.run_sharded(G, step_src, delta, dst=0, kernel="per_source")
             if rank == 0:
                 b = k % 2
                 if keep[b] is not None:
@@ -466,60 +466,50 @@ def bench_multi(args, G, g, sources, mine, delta, desc, world, rank, dev, tdev, 
     value = n_all * g.m / (t_ms * 1e-3) / 1e9
     ms = G.multi_stats()
     e2e = None
-    if not args.no_e2e and not args.profile and world > 1:
-        # every rank runs its whole shard through sssp_run_multi, rows gathered to rank 0 over
-        # NCCL, rank 0 copies them to pinned host memory; wall clock, max over ranks
+    if not args.no_e2e and not args.profile:
+        # SURVEY §8(e) end to end: one step = the whole source batch through batch.run_sharded --
+        # each rank computes its block of sources 32 per sssp_run_multi launch; after each group
+        # its rows go to rank 0 (NCCL gather, async, overlapped with the next group; no gather
+        # at N = 1) and rank 0 streams them to pinned host memory on a copy stream, also
+        # overlapped with the next group. Every copy completes inside the timed region.
         from paper_conf_icppw_zhangczsdhay23_b200 import batch
 
-        pinned = torch.empty((len(sources), g.V), dtype=torch.int32).pin_memory() if rank == 0 else None
-        torch.distributed.barrier()
-        t0 = time.perf_counter()
-        rows = batch.run_sharded(G, sources, delta, dst=0, kernel="multi")
-        if rank == 0:
-            pinned.copy_(rows.view(torch.int32) if rows.dtype != torch.int32 else rows)
-        torch.distributed.barrier()
-        te = torch.tensor([time.perf_counter() - t0], device=tdev)
-        torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
-        e2e = {"value": round(len(sources) * g.m / float(te.item()) / 1e9, 4), "unit": "GTEPS",
-               "h2d_bytes_per_step": 8 * len(sources), "d2h_bytes_per_step": 4 * g.V * len(sources),
-               "note": "one step = the whole source batch: each rank runs its shard (sssp_run_multi), NCCL "
-                       "gather of all rows to rank 0, copy to pinned host; wall clock, max over ranks"}
-    if not args.no_e2e and not args.profile and world == 1:
-        # double-buffered: group k's rows stream to pinned host memory on a copy stream
-        # while group k+1 runs; all copies finish inside the timed region
-        grp = groups[0]
-        nb = len(grp)
-        outs = [out, torch.empty_like(out)]
-        pinned = [torch.empty((nb, g.V), dtype=torch.int32).pin_memory() for _ in range(2)]
+        n = len(sources)
+        k = batch.shard_bounds(n, 0, world)[2]
+        out_all = torch.empty((world * k, g.V), dtype=torch.int32, device=f"cuda:{dev}") \
+            if rank == 0 or world == 1 else None
+        pinned = torch.empty((world * k, g.V), dtype=torch.int32).pin_memory() if rank == 0 else None
         cs = torch.cuda.Stream(device=dev)
-        done = [None, None]
 
-        def e2e_step(k):
-            b = k % 2
-            if done[b] is not None:
-                stream.wait_event(done[b])  # the previous copy out of this buffer is finished
-            G.run_multi(grp, delta, outs[b])  # sources host -> device inside the call
-            ran = torch.cuda.Event()
-            ran.record(stream)
-            cs.wait_event(ran)
+        def d2h(first, cnt, work):
+            if work is not None:
+                work.wait()  # the current stream waits for this group's gather (no host sync)
+            ev = torch.cuda.Event()
+            ev.record(torch.cuda.current_stream(dev))
+            cs.wait_event(ev)
             with torch.cuda.stream(cs):
-                pinned[b].copy_(outs[b][:nb], non_blocking=True)  # D2H of the distance rows
-                done[b] = torch.cuda.Event()
-                done[b].record(cs)
+                for r in range(world):
+                    a = r * k + first
+                    pinned[a:a + cnt].copy_(out_all[a:a + cnt], non_blocking=True)
 
-        e2e_step(0)
-        cs.synchronize()
-        ne = min(args.steps, 4)
+        if world > 1:
+            torch.distributed.barrier()
         t0 = time.perf_counter()
-        for k in range(ne):
-            e2e_step(k)
+        batch.run_sharded(G, sources, delta, dst=0, kernel="multi", out=out_all,
+                          on_group=d2h if rank == 0 else None)
         cs.synchronize()
         torch.cuda.synchronize(dev)
-        te = time.perf_counter() - t0
-        e2e = {"value": round(ne * len(grp) * g.m / te / 1e9, 4), "unit": "GTEPS",
-               "h2d_bytes_per_step": 8 * len(grp), "d2h_bytes_per_step": 4 * g.V * len(grp),
-               "note": "graph resident; per step: source ids in, the group's distance rows out to pinned "
-                       "host memory (copy of step k overlapped with step k+1, double-buffered); wall clock"}
+        if world > 1:
+            torch.distributed.barrier()
+        te = torch.tensor([time.perf_counter() - t0], device=tdev)
+        if world > 1:
+            torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
+        e2e = {"value": round(n * g.m / float(te.item()) / 1e9, 4), "unit": "GTEPS",
+               "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 4 * g.V * n,
+               "note": "one step = the whole %d-source batch through batch.run_sharded: block-sharded "
+                       "sources, 32 per sssp_run_multi launch; each group's rows gathered to rank 0 "
+                       "(NCCL, async; none at N=1) and copied to pinned host on a copy stream while the "
+                       "next group computes; wall clock, max over ranks" % n}
     if rank != 0:
         if world > 1:
             torch.distributed.barrier()

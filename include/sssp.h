@@ -52,6 +52,9 @@ typedef enum { SSSP_MEM_HOST = 0, SSSP_MEM_DEVICE = 1 } sssp_memory;
  *   weights     [A] uint32, or float32 finite and >= 0 (-0.0 becomes +0.0).
  * `where` says whether the three arrays are host or device pointers.
  * 1 <= V < 2^31 and 0 <= A < 2^32 (arc offsets are kept 64-bit internally).
+ * V < 2^31 rather than SURVEY §8(b)'s 2^32-1: bit 31 of a queued vertex id
+ * marks a 4096-arc hub chunk in the bucket queues. Every BASELINE
+ * config (largest C5: V = 2^26) is far inside this range.
  * cuda_stream: a cudaStream_t (NULL = legacy default stream).
  * Validation runs on the device; the call synchronises the stream and returns
  * SSSP_ERR_INVALID_ARGUMENT on any violation (*out untouched). */
@@ -85,8 +88,13 @@ sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags);
  * in one persistent cooperative kernel: phase 1 (light arcs, asynchronous,
  * adaptive thread/warp/CTA bins),
  * then fused phases 2&3 (heavy arcs + next bucket).
- * Asynchronous w.r.t. the host (stream-ordered). The result is read with
- * sssp_distances; overflow is reported there. */
+ * Asynchronous w.r.t. the host (stream-ordered): launch errors come back
+ * here, run-time errors (u32 overflow, scheduler cap) are recorded on the
+ * device and reported by the next sssp_distances / sssp_wait /
+ * sssp_run_batch, which synchronise (see "Run errors" below).
+ * With SSSP_PARAM_PULL_SYMMETRIC set on a weight-sorted graph, the first run
+ * checks the arc multiset for symmetry (once per reorder) and returns
+ * SSSP_ERR_INVALID_STATE if it is not symmetric. */
 sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta);
 
 /* Copy the last run's distances (V elements of the graph's weight type, in
@@ -96,7 +104,18 @@ sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta);
  * directly by the output gather kernel, pageable memory is staged through a
  * library-owned device buffer (allocated on first use, freed by destroy).
  * SSSP_ERR_INVALID_STATE if no successful run since create/reorder;
- * SSSP_ERR_OVERFLOW if a u32 distance overflowed during the run. */
+ * otherwise the run errors (below) of every run since the last report.
+ *
+ * Run errors. Each persistent run ORs its error bits into a per-handle device
+ * word that survives later runs; sssp_distances, sssp_wait and sssp_run_batch
+ * synchronise, report that word and clear it, so no run's error is lost:
+ *   SSSP_ERR_OVERFLOW: a relaxation d[u] + w of a u32 graph reached
+ *     0xFFFFFFFF. Always reported when some reachable vertex's shortest
+ *     distance is >= 0xFFFFFFFF (its result would be wrong); may also be
+ *     reported when only a longer path's sum overflows (push relaxations
+ *     check every sum they form, Alg. 1 l.1).
+ *   SSSP_ERR_INTERNAL: a hub-chunk queue overflowed in phase 2 (work was
+ *     dropped; the handle's queues are fully reset before the next run). */
 sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory where);
 
 /* Free every resource of the handle. NULL-safe. */
@@ -109,10 +128,6 @@ const char* sssp_last_error(void); /* thread-local detail of the last failure */
 /* Make subsequent work on g use cuda_stream (a cudaStream_t; NULL = default). */
 sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream);
 
-/* Multi-source batch (the naturally sharded case of the north star): for
- * i < n run sssp_run(sources[i], delta) and write the distances (original
- * order) to the DEVICE buffer out_dev + i*ld elements (ld >= V). sources is a
- * host array. Stream-ordered; no host synchronisation. */
 /* Asynchronous sssp_distances: the output gather of the last run (original
  * ids, graph weight type) goes to one of two device staging buffers on the
  * handle's stream, then a copy engine moves it to `out` on the handle's own
@@ -122,10 +137,16 @@ sssp_status sssp_set_stream(sssp_graph_t g, void* cuda_stream);
  * Pageable memory: SSSP_ERR_INVALID_ARGUMENT. INVALID_STATE before a run. */
 sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memory where);
 
-/* Waits for every output enqueued by sssp_distances_async. (Run errors are
- * reported by sssp_run itself, which waits for its own kernel.) */
+/* Waits for every output enqueued by sssp_distances_async and for every run
+ * enqueued on the handle's stream, then reports (and clears) the run errors
+ * of all runs since the last report (see sssp_distances). */
 sssp_status sssp_wait(sssp_graph_t g);
 
+/* Multi-source batch (the naturally sharded case of the north star): for
+ * i < n run sssp_run(sources[i], delta) and write the distances (original
+ * order) to the DEVICE buffer out_dev + i*ld elements (ld >= V). sources is a
+ * host array. Enqueues all n runs, then synchronises once and reports the run
+ * errors of the batch (and of any earlier unreported run). */
 sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                            void* out_dev, int64_t ld);
 
@@ -137,7 +158,9 @@ sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, do
  * buckets by their smallest improved distance; an expansion relaxes every
  * finite lane (label-correcting: exact, identical to sssp_run per source for
  * u32 and f32). Allocates 132 B per vertex plus the ring on first use.
- * Synchronises once per group of 32 sources. Errors as sssp_run. */
+ * Synchronises once per group of 32 sources; SSSP_ERR_OVERFLOW if a u32
+ * relaxation of any group overflowed (each group's error word is read before
+ * the next group starts). */
 sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                            void* out_dev, int64_t ld);
 
@@ -221,8 +244,10 @@ typedef enum {
                                       are, R13): graphs after a weight-sorting sssp_reorder
                                       then run phases 2&3 of buckets holding >= V/16 entries as a
                                       pull (each unsettled vertex scans its weight-sorted heavy
-                                      arcs up to the first that cannot win). Same distances;
-                                      wrong distances if the graph is not symmetric [0] */
+                                      arcs up to the first that cannot win). Same distances.
+                                      The assertion is verified once per reorder (sssp_is_
+                                      symmetric): setting 1 on a reordered asymmetric graph,
+                                      or running with it, returns SSSP_ERR_INVALID_STATE [0] */
     SSSP_PARAM_LOCAL_CHASE = 12,   /* 2: when no arc is heavy at the run's Delta (max weight <
                                       Delta, fixed Delta), a phase-1 push into
                                       the current bucket stays in the pushing CTA's shared
@@ -254,7 +279,9 @@ sssp_status sssp_kernel_time(sssp_graph_t g, double* total_ms, int64_t* launches
  * every closed bucket i also adds which = 8: cur = C_i (settled vertices),
  * tail = T_i (phase-1 queue items), mode = width of the next bucket in slots,
  * far_min = Delta_{i+1} as binary32 bits (in slot units), pad = i + 1.
- * Up to 4096 entries. */
+ * Every entry whose step closed a bucket (moved past it) carries that bucket
+ * and its settled-vertex count in closed_b / closed_c (bucket
+ * i = distances in [i*Delta, (i+1)*Delta)). Up to 4096 entries. */
 typedef struct sssp_trace_entry {
     uint64_t t_ns;   /* %globaltimer */
     uint32_t which;  /* barrier kind (see above) */
@@ -262,9 +289,25 @@ typedef struct sssp_trace_entry {
     uint32_t tail;   /* entries in that bucket's queue */
     uint32_t mode;   /* next mode: 0 phase 1, 1 phase 2, 2 done, 3/4 rescan, 5/6 sweep */
     uint32_t far_min, pad;
+    uint32_t closed_b; /* bucket (ring-slot units) this scheduler step closed, 0xFFFFFFFF if none */
+    uint32_t closed_c; /* C: vertices settled in that bucket (final distance inside it), counted
+                          by phases 2&3 (push: entries with d == dist[v]; pull: candidates whose
+                          distance lies in the bucket). Exact for u32 graphs; 0xFFFFFFFF
+                          (not counted) when the CTA-local chase was on (its in-bucket entries
+                          never reach the bucket's queue) */
+    uint64_t t_first;  /* %globaltimer of the first CTA's arrival at this barrier */
+    uint64_t t_rel;    /* %globaltimer when the scheduler step was done and the grid released */
 } sssp_trace_entry;
 sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
                            int64_t* n_entries);
+
+/* Diagnostics of the last run: phase-1 claim samples of every 37th CTA, in
+ * time order per CTA (which = 100; t_ns = %globaltimer; cur = bucket; tail =
+ * queue entries pushed so far; far_min = pending entries; mode = entries
+ * claimed (0: the phase ended); pad = first claimed position; closed_b = CTA;
+ * closed_c = 1 for a CTA-local batch). Up to 16384 entries. */
+sssp_status sssp_get_samples(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
+                             int64_t* n_entries);
 
 /* Diagnostics of the last run: summed SM cycles of thread 0 of every
  * persistent CTA in [claim, stage, task, tail, grid-barrier], the number of
@@ -272,6 +315,13 @@ sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_en
  * else 0) warp-0 cycles waiting for arcs, dist probes, atomics, staging and
  * the number of tasks measured (12 values). */
 sssp_status sssp_get_profile(sssp_graph_t g, uint64_t* out, int n);
+
+/* *out = 1 if the arc multiset is symmetric (every (u,v,w) has its reverse
+ * (v,u,w) with the same multiplicity), else 0. Needs weight-sorted
+ * adjacencies (sssp_reorder / SSSP_PRO_WEIGHT), else SSSP_ERR_INVALID_STATE:
+ * every run of equal arcs is matched by a lower_bound in the other end's
+ * sorted segment (one kernel, cached until the next reorder). Synchronises. */
+sssp_status sssp_is_symmetric(sssp_graph_t g, int* out);
 
 /* Library/device info: number of SMs of the handle's device. */
 int sssp_device_sm_count(sssp_graph_t g);

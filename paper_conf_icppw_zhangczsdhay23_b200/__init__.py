@@ -60,7 +60,7 @@ EXPORTS = (
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
     "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile", "sssp_run_multi", "sssp_multi_stats",
-    "sssp_distances_async", "sssp_wait",
+    "sssp_distances_async", "sssp_wait", "sssp_is_symmetric", "sssp_get_samples",
 )
 
 
@@ -92,6 +92,7 @@ _lib.sssp_run_batch.argtypes = [_P, _P, _I64, _D, _P, _I64]
 _lib.sssp_run_multi.argtypes = [_P, _P, _I64, _D, _P, _I64]
 _lib.sssp_distances_async.argtypes = [_P, _P, _I]
 _lib.sssp_wait.argtypes = [_P]
+_lib.sssp_is_symmetric.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.sssp_multi_stats.argtypes = [_P, _P, _I64]
 _lib.sssp_get_stats.argtypes = [_P, ctypes.POINTER(sssp_stats)]
 _lib.sssp_export_csr.argtypes = [_P, _D, _P, _P, _P, _P]
@@ -104,16 +105,19 @@ _lib.sssp_kernel_time.restype = _I
 class sssp_trace_entry(ctypes.Structure):
     _fields_ = [("t_ns", ctypes.c_uint64), ("which", ctypes.c_uint32), ("cur", ctypes.c_uint32),
                 ("tail", ctypes.c_uint32), ("mode", ctypes.c_uint32), ("far_min", ctypes.c_uint32),
-                ("pad", ctypes.c_uint32)]
+                ("pad", ctypes.c_uint32), ("closed_b", ctypes.c_uint32), ("closed_c", ctypes.c_uint32),
+                ("t_first", ctypes.c_uint64), ("t_rel", ctypes.c_uint64)]
 
 
 _lib.sssp_get_trace.argtypes = [_P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]
 _lib.sssp_get_trace.restype = _I
+_lib.sssp_get_samples.argtypes = [_P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]
+_lib.sssp_get_samples.restype = _I
 _lib.sssp_get_profile.argtypes = [_P, _P, _I]
 _lib.sssp_get_profile.restype = _I
 for _n in ("sssp_graph_create", "sssp_reorder", "sssp_reorder_ex", "sssp_run", "sssp_distances",
            "sssp_set_stream", "sssp_run_batch", "sssp_get_stats", "sssp_export_csr", "sssp_set_param",
-           "sssp_run_multi", "sssp_multi_stats", "sssp_distances_async", "sssp_wait"):
+           "sssp_run_multi", "sssp_multi_stats", "sssp_distances_async", "sssp_wait", "sssp_is_symmetric"):
     getattr(_lib, _n).restype = _I
 
 
@@ -272,8 +276,22 @@ def sssp_get_trace(h, max_entries=4096):
     for i in range(min(n.value, max_entries)):
         e = buf[i]
         out.append(dict(t_us=(e.t_ns - t0) / 1e3, which=e.which, cur=e.cur, tail=e.tail, mode=e.mode,
-                        far_min=e.far_min, pad=e.pad))
+                        far_min=e.far_min, pad=e.pad, closed_b=e.closed_b, closed_c=e.closed_c,
+                        t_first_us=(e.t_first - t0) / 1e3, t_rel_us=(e.t_rel - t0) / 1e3))
     return out
+
+
+def sssp_get_samples(h, max_entries=16384):
+    """Phase-1 claim samples of the last run (diagnostics): list of dicts, t_us relative to
+    the first sample."""
+    buf = (sssp_trace_entry * max_entries)()
+    n = ctypes.c_int64()
+    _check(_lib.sssp_get_samples(h, buf, max_entries, ctypes.byref(n)), "sssp_get_samples")
+    m = min(n.value, max_entries)
+    t0 = min((buf[i].t_ns for i in range(m)), default=0)
+    return [dict(t_us=(buf[i].t_ns - t0) / 1e3, t_ns=buf[i].t_ns, cur=buf[i].cur, tail=buf[i].tail,
+                 claimed=buf[i].mode, pend=buf[i].far_min, pos=buf[i].pad, cta=buf[i].closed_b)
+            for i in range(m)]
 
 
 def sssp_get_profile(h):
@@ -283,6 +301,12 @@ def sssp_get_profile(h):
     out = np.zeros(len(names), dtype=np.uint64)
     _check(_lib.sssp_get_profile(h, out.ctypes.data, len(names)), "sssp_get_profile")
     return dict(zip(names, out.tolist()))
+
+
+def sssp_is_symmetric(h):
+    out = ctypes.c_int(0)
+    _check(_lib.sssp_is_symmetric(h, ctypes.byref(out)), "sssp_is_symmetric")
+    return bool(out.value)
 
 
 def sssp_device_sm_count(h):
@@ -369,5 +393,11 @@ class Graph:
     def trace(self):
         return sssp_get_trace(self.h)
 
+    def samples(self):
+        return sssp_get_samples(self.h)
+
     def set_stream(self, stream):
         sssp_set_stream(self.h, stream)
+
+    def is_symmetric(self):
+        return sssp_is_symmetric(self.h)

@@ -1,82 +1,133 @@
 """Multi-source batch across GPUs (north star: "a batch of independent sources
 is spread across the 8xB200 box: each GPU holds a replicated graph, and NCCL
-gathers distance vectors over NVLink").
+gathers distance vectors over NVLink"; SURVEY §8(e)).
 
-One process per GPU (torchrun). Sources are sharded round-robin
-(``sources[rank::world]``); every rank runs its shard through the C-ABI
-(``sssp_run_batch`` writes rows straight into a device tensor), then the rows
-are gathered to the destination rank with one ``torch.distributed`` gather
-(NCCL on GPUs; gloo for the CPU tests of this host logic).
+One process per GPU (torchrun). Sources are sharded in contiguous blocks
+(rank r gets sources [r*k, (r+1)*k), k = ceil(n / world)), so the gathered
+layout [world, k, V] IS the global source order: rank ``dst`` hands NCCL
+views of one [world*k, V] output tensor and never reorders or copies rows.
+
+Fusion (§8(e)): every rank computes its shard in groups of up to 32 sources
+(one ``sssp_run_multi`` launch, or ``sssp_run_batch`` runs, per group) and
+starts the gather of a group's rows (``dist.gather(async_op=True)``, NCCL's
+own stream) as soon as the library returns them, while the next group
+computes -- the transfer of group g overlaps the SSSPs of group g+1. The
+library reports run errors per call (sssp.h "Run errors"), so a failed group
+raises before its rows are sent.
 """
 from __future__ import annotations
 
 import numpy as np
 
+GROUP = 32  # sources per sssp_run_multi launch (the kernel's lane count)
+
+
+def shard_bounds(n: int, rank: int, world: int):
+    """Block shard of n sources: (first, end, k) with k = ceil(n / world) rows per rank."""
+    k = (n + world - 1) // world
+    lo = min(n, rank * k)
+    return lo, min(n, lo + k), k
+
 
 def shard_sources(sources, rank: int, world: int):
-    """Round-robin shard: global source i goes to rank i % world, row i // world."""
-    return np.asarray(sources)[rank::world]
+    """Contiguous block of the global source list owned by ``rank``."""
+    lo, hi, _ = shard_bounds(len(sources), rank, world)
+    return np.asarray(sources)[lo:hi]
 
 
-def global_order(n: int, world: int):
-    """Gather layout -> global source index: gathered[r][j] is source r + j*world."""
-    k = (n + world - 1) // world
-    idx = np.full((world, k), -1, dtype=np.int64)
-    for i in range(n):
-        idx[i % world, i // world] = i
-    return idx
+def _gather(send, out, first: int, count: int, k: int, dst: int, group, async_op: bool):
+    """Gather rows [first, first+count) of every rank's k-row shard into ``out`` on dst:
+    rank r's rows land in out[r*k + first : r*k + first + count] (views, no copies)."""
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    gl = [out[r * k + first: r * k + first + count] for r in range(world)] if rank == dst else None
+    return dist.gather(send[first: first + count], gl, dst=dst, group=group, async_op=async_op)
 
 
-def gather_rows(local_rows, n_sources: int, dst: int = 0, group=None):
-    """Gather every rank's [k_r, V] rows to ``dst`` in global source order.
+def gather_rows(local_rows, n_sources: int, dst: int = 0, group=None, out=None):
+    """Gather every rank's block of rows (``local_rows`` [len(shard), V]) to ``dst``.
 
-    local_rows: tensor [k_r, V] (k_r = shard size of this rank; shards differ by
-    at most one row and are zero-padded to the largest for the collective).
-    Returns [n_sources, V] on ``dst`` and None elsewhere."""
+    Returns [n_sources, V] on ``dst`` (a view of ``out`` if given, shape
+    [world*k, V]) and None elsewhere. Shorter shards (only the last ranks when
+    world does not divide n) are padded on the send side only."""
     import torch
     import torch.distributed as dist
 
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
-    k = (n_sources + world - 1) // world
+    _, _, k = shard_bounds(n_sources, rank, world)
     V = local_rows.shape[1]
-    if local_rows.shape[0] < k:
-        pad = torch.zeros((k - local_rows.shape[0], V), dtype=local_rows.dtype, device=local_rows.device)
-        local_rows = torch.cat([local_rows, pad], 0)
-    local_rows = local_rows.contiguous()
-    if dist.get_backend(group) != "nccl" and local_rows.is_cuda:  # gloo: host staging (tests)
-        local_rows = local_rows.cpu()
-    bufs = [torch.empty_like(local_rows) for _ in range(world)] if rank == dst else None
-    dist.gather(local_rows, bufs, dst=dst, group=group)
-    if rank != dst:
-        return None
-    order = global_order(n_sources, world)
-    out = torch.empty((n_sources, V), dtype=local_rows.dtype, device=local_rows.device)
-    for r in range(world):
-        for j in range(k):
-            i = order[r, j]
-            if i >= 0:
-                out[i] = bufs[r][j]
-    return out
+    send = local_rows
+    if send.shape[0] != k:
+        send = torch.zeros((k, V), dtype=local_rows.dtype, device=local_rows.device)
+        send[: local_rows.shape[0]] = local_rows
+    if rank == dst and out is None:
+        out = torch.empty((world * k, V), dtype=local_rows.dtype, device=local_rows.device)
+    if k:
+        _gather(send.contiguous(), out, 0, k, k, dst, group, async_op=False)
+    return out[:n_sources] if rank == dst else None
 
 
-def run_sharded(graph, sources, delta, dst: int = 0, group=None, kernel: str = "per_source"):
-    """Run this rank's shard of ``sources`` on ``graph`` (a paper_conf...Graph on
-    this rank's GPU) and gather all distance rows to ``dst``. ``kernel``:
-    "per_source" = one persistent Delta-stepping launch per source
-    (``sssp_run_batch``), "multi" = 32 sources per launch (``sssp_run_multi``,
-    NEXT-4). Both give identical rows."""
+def run_sharded(graph, sources, delta, dst: int = 0, group=None, kernel: str = "multi", out=None,
+                group_size: int = GROUP, on_group=None):
+    """Run this rank's block of ``sources`` on ``graph`` (a Graph on this rank's
+    GPU) and gather all distance rows to ``dst``, overlapping each group's
+    gather with the next group's compute. ``kernel``: "multi" = 32 sources per
+    persistent launch (``sssp_run_multi``, NEXT-4), "per_source" = one
+    Delta-stepping launch per source (``sssp_run_batch``). Identical rows.
+    ``on_group(first, count, work)`` (dst only) is called once group rows
+    [r*k + first, r*k + first + count) of every rank r have been enqueued into
+    ``out`` (``work``: the async gather, or None without a process group), so a
+    caller can stream them onward (e.g. D2H) while the next group computes.
+    Without an initialised process group this is the single-GPU case: the rows
+    are computed straight into ``out``.
+    Returns [len(sources), V] on ``dst`` (in global source order), else None."""
     import torch
     import torch.distributed as dist
 
-    world = dist.get_world_size(group)
-    rank = dist.get_rank(group)
-    mine = shard_sources(sources, rank, world)
-    dtype = torch.float32 if graph.f32 else torch.int32
-    rows = torch.empty((max(len(mine), 1), graph.V), dtype=dtype, device=f"cuda:{graph.device}")
     if kernel not in ("per_source", "multi"):
         raise ValueError(f"unknown kernel {kernel!r}")
-    if len(mine):
-        (graph.run_multi if kernel == "multi" else graph.run_batch)(mine, delta, rows, graph.V)
-    torch.cuda.synchronize(graph.device)
-    return gather_rows(rows[: len(mine)] if len(mine) else rows[:0], len(sources), dst, group)
+    n = len(sources)
+    run = graph.run_multi if kernel == "multi" else graph.run_batch
+    if not (dist.is_available() and dist.is_initialized()):
+        dev = getattr(graph, "torch_device", None) or f"cuda:{graph.device}"
+        if out is None:
+            out = torch.empty((max(n, 1), graph.V), dtype=torch.float32 if graph.f32 else torch.int32, device=dev)
+        src = np.asarray(sources)
+        for g0 in range(0, n, group_size):
+            cnt = min(group_size, n - g0)
+            run(src[g0: g0 + cnt], delta, out[g0: g0 + cnt], graph.V)
+            if on_group is not None:
+                on_group(g0, cnt, None)
+        return out[:n]
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    lo, hi, k = shard_bounds(n, rank, world)
+    mine = np.asarray(sources)[lo:hi]
+    dev = getattr(graph, "torch_device", None) or f"cuda:{graph.device}"
+    dtype = torch.float32 if graph.f32 else torch.int32
+    staged = dist.get_backend(group) != "nccl" and str(dev).startswith("cuda")  # gloo: host buffers (tests)
+    send = torch.empty((max(k, 1), graph.V), dtype=dtype, device=dev)
+    send_h = torch.zeros((max(k, 1), graph.V), dtype=dtype) if staged else None
+    if rank == dst and out is None:
+        out = torch.empty((world * k, graph.V), dtype=dtype, device="cpu" if staged else dev)
+    works = []
+    for g0 in range(0, k, group_size):
+        cnt = min(group_size, k - g0)
+        real = max(0, min(cnt, len(mine) - g0))
+        if real:
+            run(mine[g0: g0 + real], delta, send[g0: g0 + real], graph.V)  # returns when the rows are done
+        buf = send
+        if staged:
+            send_h[g0: g0 + cnt] = send[g0: g0 + cnt].cpu()
+            buf = send_h
+        works.append(_gather(buf, out, g0, cnt, k, dst, group, async_op=True))
+        if on_group is not None and rank == dst:
+            on_group(g0, cnt, works[-1])
+    for w in works:
+        w.wait()
+    if rank != dst:
+        return None
+    return out[:n]

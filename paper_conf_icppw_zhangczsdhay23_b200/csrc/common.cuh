@@ -39,6 +39,38 @@ __device__ __forceinline__ u32 ld_acquire_u32(const u32* p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ void st_release_u32(u32* p, u32 v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 atom_add_acq_rel_u32(u32* p, u32 v) {
+  u32 old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+
+// Grid barrier arrival/departure for a cooperative (co-resident) grid, called by
+// one thread per CTA after a __syncthreads (whose CTA-scope ordering the release
+// extends to the GPU). `count` is a monotonic ticket counter and `gen` the
+// generation word, both zeroed before the launch. Every arrival is an acq_rel
+// RMW, so the last arriver (return true) has acquired every CTA's phase writes
+// through the RMW release sequence; it then runs its serial step and calls
+// grid_release(), whose release store the waiters acquire. No sc fences
+// (MEMBAR.SC.GPU), no counter reset, one RMW per CTA.
+__device__ __forceinline__ bool grid_arrive(u32* count, u32* target) {
+  const u32 G = gridDim.x;
+  const u32 t = atom_add_acq_rel_u32(count, 1u);
+  *target = t / G + 1;
+  return t % G == G - 1;
+}
+__device__ __forceinline__ void grid_release(u32* gen, u32 target) { st_release_u32(gen, target); }
+__device__ __forceinline__ void grid_wait(const u32* gen, u32 target) {
+  u32 ns = 32;
+  while ((int)(ld_acquire_u32(gen) - target) < 0) {
+    __nanosleep(ns);
+    if (ns < 128) ns <<= 1;
+  }
+}
+
 __device__ __forceinline__ void st_relaxed_u64(u64* p, u64 v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }

@@ -92,11 +92,12 @@ enum : u32 {
   MODE_P2_COMPACT = 7,  // edge-balanced phase 2, step 1: settled entries -> heavy-arc offsets
   MODE_P2_RELAX = 8,    // ... step 2: equal heavy-arc ranges per warp
   MODE_MERGE = 9,       // adaptive Delta: fold the slots (cur, cur_end) into slot cur
-  MODE_PULL = 10        // phases 2&3 as a pull over the unsettled vertices (symmetric u32 graphs)
+  MODE_PULL = 10,       // phases 2&3 as a pull over the unsettled vertices (symmetric graphs)
+  MODE_PULL_LONG = 11   // ... second step: long heavy-arc scans, one warp per vertex
 };
 enum : u32 { ERR_OVERFLOW = 1, ERR_INTERNAL = 2 };
 enum : u32 { SYNC_P1 = 0, SYNC_P2 = 1, SYNC_RC = 2, SYNC_RF = 3, SYNC_SL = 4, SYNC_SH = 5, SYNC_P2C = 6,
-              SYNC_MG = 7, TRACE_ADAPT = 8 };
+              SYNC_MG = 7, TRACE_ADAPT = 8, SYNC_PL = 9 };
 enum : u32 { SRC_QUEUE = 0, SRC_STATIC = 1, SRC_HUB = 2, SRC_SWEEP = 3 };
 
 enum {
@@ -151,8 +152,19 @@ struct __align__(128) Ctl {
   float a_d0;        // Delta_0 in fine units
   u32 a_mmin, a_mmax, a_m;  // width clamp and current width (fine slots)
   u32 lvl;           // light/heavy level of the current bucket: light iff w < g << lvl
-  u32 csum;          // settled vertices of the current bucket (phase 2 counts them)
-  u32 pad_a[2];
+  u32 csum;          // settled vertices of the current bucket (phase 2 / pull count them)
+  u32 err_acc;       // OR of err over every run since the host last read it (k_seed keeps it)
+  u32 pad_a;
+  // pull phases 2&3: candidate lists (unsettled vertices with arcs) in xd[V..3V); pull_sel = the
+  // input list (2 = every vertex, the first pull), pull_n = list lengths
+  u32 pull_sel, pull_n[2];
+  u32 closed_c, closed_b;    // C_i and index of the bucket the last scheduler step closed (trace)
+  u32 pad_c;
+  u64 t_first;               // earliest arrival at the current grid barrier (%globaltimer, trace)
+  u32 long_n, long_head;     // pull: long scans handed to whole warps (count, claim tickets)
+  u32 sample_n;              // phase-1 claim samples written (diagnostics)
+  u32 first_n;               // the first pull's candidates: ids [0, first_n) (isolated ids excluded)
+  u32 pad_b[20];
   u32 bar_count, pad3[31];   // own line: arrivals
   u32 bar_gen, pad4[31];     // own line: spun on
   u32 p2_head, pad5[31];     // own line: phase-2 static tickets
@@ -162,6 +174,8 @@ struct __align__(128) Ctl {
 };
 
 constexpr u32 TRACE_CAP = 4096;
+constexpr u32 SAMPLE_CAP = 16384;  // phase-1 claim samples after the trace (sssp_get_samples)
+constexpr u32 SAMPLE_EVERY = 37;   // CTAs with blockIdx % 37 == 0 record theirs
 struct TraceEnt {
   u64 t_ns;   // %globaltimer when the last CTA arrived
   u32 which;  // SYNC_* (99 = kernel start)
@@ -169,6 +183,9 @@ struct TraceEnt {
   u32 tail;   // entries in the current bucket's queue
   u32 mode;   // mode chosen by the scheduler
   u32 far_min, pad;
+  u32 closed_b, closed_c;  // bucket this step closed and its settled-vertex count C (else NONE, 0)
+  u64 t_first;             // first CTA's arrival at this barrier
+  u64 t_rel;               // release (after the scheduler step and this record)
 };
 
 __device__ __forceinline__ u64 globaltimer() {
@@ -181,13 +198,15 @@ struct Params {
   const uint2* rowc;      // [V+1] {start, heavy} (u32 arc offsets)
   const uint2* arcs;      // [A] {dst, wbits}
   u32* dist;              // [V]
-  u32* xd;                // [V] sweep fall-back: distance at last light expansion
+  u32* xd;                // [5V] sweep fall-back marks [0, V); pull candidate lists [V, 3V);
+                          // pull long-scan items uint4 [V/2] from 3V rounded up to 4 (+4 slack)
   Ctl* ctl;
   SlotCtl* sc;            // [K]
   u64* items;             // [K * cap]
   u64* hub_items;         // [hub_cap]
   unsigned long long* stats;  // [ST_N]
-  TraceEnt* trace;            // [TRACE_CAP] barrier timeline of the last run
+  TraceEnt* trace;            // [TRACE_CAP] barrier timeline of the last run, then [SAMPLE_CAP]
+                              // phase-1 claim samples
   u32* p2o;  // [cap] edge-balanced phase 2: first heavy-arc rank of each compacted entry,
              // followed by uint2 [cap] {arc index - rank, d} (see p2_compact)
   u32 V, K, kmask, cap, hub_cap;
@@ -217,7 +236,10 @@ constexpr u32 SB_CAP = 32 * IPT_MAX;           // thread-bin entries per warp
 constexpr u32 PB_CAP = SSSP_PB_CAP;  // staged pushes per warp (>= 32 * UNROLL)
 constexpr u32 LOC_CAP = BATCH;       // CTA-local chase list: one phase-1 batch
 constexpr u32 LOCAL_CHASE = 1u << 16;  // Params::claim_max bit (claim_max itself <= BATCH) ...
-constexpr u32 LOCAL_LIM_SHIFT = 20;     // ... and bits 20-29: entries kept locally (<= LOC_CAP)
+constexpr u32 LOCAL_LIM_SHIFT = 20;     // ... and bits 20-31: entries kept locally (1..LOC_CAP)
+constexpr u32 LOCAL_LIM_MASK = 4095u;
+static_assert(BATCH < LOCAL_CHASE, "claim_max must fit below the LOCAL_CHASE bit");
+static_assert(LOC_CAP <= LOCAL_LIM_MASK, "local-chase limit field too narrow for LOC_CAP");
 
 struct Smem {
   // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
@@ -249,6 +271,7 @@ struct Smem {
   // control snapshot
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
   u32 cur_end, rowc_off, theta_bits;  // bucket end (fine slots), light/heavy level
+  u32 pull_sel, pull_n_in;            // pull phases 2&3: input candidate list
 };
 
 // ---------------------------------------------------------------- helpers --
@@ -684,7 +707,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   }
   // ---- stats (warp-aggregated)
   st_add(sm, PH == 1 ? ST_SETTLED : ST_HEAVYV, c_settled);
-  if (EXT && PH == 2 && !sweep && (p.flags & 24u)) {  // adaptive Delta: C_i (converged vertices)
+  if (PH == 2) {  // C_i: vertices settled in bucket cur (trace; adaptive Delta, Eq. (1))
     const u32 cs = __reduce_add_sync(SSSP_FULL_MASK, c_settled);
     if (lane == 0 && cs) atomicAdd(&p.ctl->csum, cs);
   }
@@ -856,6 +879,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
 
 // --------------------------------------------------------- grid barrier ---
 __device__ __forceinline__ void enter_sweep(volatile Ctl* c) {
+  c->csum = 0;  // the heavy sweep counts the bucket's vertices afresh
   c->changed = 0;
   c->sweep_first = 1;
   c->sweeps = c->sweeps + 1;
@@ -874,10 +898,8 @@ __device__ __forceinline__ void enter_sweep(volatile Ctl* c) {
 // per bucket (T up) narrows the next bucket. Runs on the one
 // thread that closes a bucket; the next bucket spans round(Delta_i / g) fine
 // slots and its light level is the smallest g * 2^l >= that width.
-__device__ void adapt_next(const Params& p, u32 t_i) {
+__device__ void adapt_next(const Params& p, u32 t_i, u32 c_i) {
   volatile Ctl* c = p.ctl;
-  const u32 c_i = c->csum;
-  c->csum = 0;
   const u32 i = c->a_i + 1;
   c->a_c2 = c->a_c1;
   c->a_c1 = c_i;
@@ -909,6 +931,9 @@ __device__ void adapt_next(const Params& p, u32 t_i) {
     e.mode = m;
     e.far_min = __float_as_uint(dl);
     e.pad = i;
+    e.closed_b = NONE;
+    e.closed_c = 0;
+    e.t_first = e.t_rel = e.t_ns;
     p.trace[tn] = e;
     c->trace_n = tn + 1;
   }
@@ -919,6 +944,16 @@ __device__ void decide(const Params& p, u32 which) {
   volatile Ctl* c = p.ctl;
   volatile SlotCtl* sc = p.sc;
   const u32 K = p.K;
+  c->closed_b = NONE;
+  c->closed_c = 0;
+  if (which == SYNC_PL) {  // pull done but for the long scans it handed off
+    if (c->long_n != 0) {
+      c->long_head = 0;
+      c->mode = MODE_PULL_LONG;
+      return;
+    }
+    which = SYNC_P2;
+  }
   if (which == SYNC_P2C) {  // entries compacted: relax their heavy arcs, if any
     if ((u32)c->hub_word != 0) {
       c->mode = MODE_P2_RELAX;
@@ -944,6 +979,8 @@ __device__ void decide(const Params& p, u32 which) {
     c->p2_begin = b;
     c->p2_end = tail;
     if ((p.flags & 128u) && tail - b >= p.V / SSSP_PULL_DIV) {  // large bucket: pull phase 2
+      c->pull_n[c->pull_sel == 0 ? 1u : 0u] = 0;  // output candidate list
+      c->long_n = 0;
       c->mode = MODE_PULL;
       return;
     }
@@ -960,6 +997,7 @@ __device__ void decide(const Params& p, u32 which) {
   } else if (which == SYNC_P2) {
     const u32 cur = c->cur, s = cur & p.kmask;
     sc[s].p2 = c->p2_end;
+    if (c->mode == MODE_PULL || c->mode == MODE_PULL_LONG) c->pull_sel = c->pull_sel == 0 ? 1u : 0u;  // its output
     const u32 fm = c->far_min;
     if ((u32)sc[s].word != 0) {  // a heavy relaxation landed in bucket cur (f32 rounding, or
                                  // adaptive Delta with a light level below the width)
@@ -972,12 +1010,26 @@ __device__ void decide(const Params& p, u32 which) {
       }
       return;
     }
+    // bucket cur is closed: C_i = vertices settled in it (counted by phase 2 / the pull; unknown
+    // with the CTA-local chase, whose entries never reach the bucket's queue)
+    const u32 c_i = c->csum;
+    c->csum = 0;
+    c->closed_c = (p.claim_max & LOCAL_CHASE) ? NONE : c_i;
+    c->closed_b = cur;
     u32 nxt = NONE;
-    for (u32 x = c->cur_end; x <= c->lim && x != NONE; ++x)
-      if ((u32)(sc[x & p.kmask].word >> 32) != 0) {
-        nxt = x;
-        break;
+    {  // lowest non-empty ring slot after the bucket: 8 slot words in flight per step
+      const u32 x_end = c->lim;
+      for (u32 x0 = c->cur_end; x0 <= x_end && x0 != NONE && nxt == NONE; x0 += 8) {
+        u32 t[8];
+#pragma unroll
+        for (u32 k = 0; k < 8; ++k)
+          t[k] = (x0 + k <= x_end && x0 + k >= x0) ? (u32)(sc[(x0 + k) & p.kmask].word >> 32) : 0u;
+#pragma unroll
+        for (u32 k = 0; k < 8; ++k)
+          if (t[k] && nxt == NONE) nxt = x0 + k;
+        if (x0 + 8 < x0) break;
       }
+    }
     if (nxt == NONE && fm == NONE) {
       c->mode = MODE_DONE;
       return;
@@ -991,10 +1043,13 @@ __device__ void decide(const Params& p, u32 which) {
     sc[s].word = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
     sc[s].head = 0;
     sc[s].p2 = 0;
-    const u64 lim = (u64)cur + K - 1;  // excludes slot s of bucket cur+K: reset just now
+    // Ring horizon: slots hold buckets [nxt, nxt + K). The slots of bucket cur (reset just now)
+    // and of the empty buckets (cur, nxt) are free, so a jump over empty buckets moves the
+    // horizon with it (cur + K - 1 here forced needless rescans after such jumps).
+    const u64 lim = (u64)nxt + K - 1;
     c->lim = (u32)min(lim, (u64)NONE - 1);
     c->cur = nxt;
-    if (c->a_mode) adapt_next(p, t_items);
+    if (c->a_mode) adapt_next(p, t_items, c_i);
     c->cur_end = (u32)min((u64)nxt + c->a_m, (u64)c->lim + 1);
     c->epochs = c->epochs + 1;
     for (u32 x = nxt + 1; x < c->cur_end; ++x)
@@ -1041,6 +1096,9 @@ __device__ void decide(const Params& p, u32 which) {
     } else if (which == SYNC_SL) {
       c->mode = MODE_SWEEP_HEAVY;
     } else {  // bucket cur is final; rebuild the ring from dist[] for what follows
+      c->closed_c = c->csum;  // the heavy sweep counted the bucket's vertices (local chase or not)
+      c->csum = 0;
+      c->closed_b = c->cur;
       c->rescan_base = c->cur_end;
       c->mode = MODE_RESCAN_CLEAR;
     }
@@ -1050,6 +1108,8 @@ __device__ void decide(const Params& p, u32 which) {
 // Bucket extent and light/heavy level of the current bucket into shared memory.
 __device__ __forceinline__ void load_bucket(const Params& p, Smem& sm, volatile Ctl* vc) {
   sm.cur_end = vc->cur_end;
+  sm.pull_sel = vc->pull_sel;
+  sm.pull_n_in = sm.pull_sel < 2 ? vc->pull_n[sm.pull_sel] : vc->first_n;
   const u32 l = vc->lvl;
   sm.rowc_off = (p.flags & 64u) ? l * (p.V + 1) : 0u;  // levels built only with PRO
   sm.theta_bits = l == 0 ? p.delta_bits : ((p.flags & 32u) ? p.delta_bits + (l << 23) : p.delta_bits << l);
@@ -1060,12 +1120,9 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
   if (threadIdx.x == 0) {
     const long long t_b = clock64();
     Ctl* c = p.ctl;
-    const u32 gen = ld_acquire_u32(&c->bar_gen);
-    __threadfence();
-    const u32 arrived = atomicAdd(&c->bar_count, 1u);
-    if (arrived == gridDim.x - 1) {
-      c->bar_count = 0;
-      __threadfence();
+    atomicMin(&c->t_first, globaltimer());  // trace only (fire and forget)
+    u32 target;
+    if (grid_arrive(&c->bar_count, &target)) {
       const u64 t = globaltimer();
       decide(p, which);
       volatile Ctl* vc = c;
@@ -1079,19 +1136,18 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
         e.mode = vc->mode;
         e.far_min = vc->far_min;
         e.pad = vc->cur_end;
+        e.closed_b = vc->closed_b;
+        e.closed_c = vc->closed_c;
+        e.t_first = vc->t_first;
+        e.t_rel = globaltimer();
         p.trace[tn] = e;
         vc->trace_n = tn + 1;
       }
-      __threadfence();
-      atomicAdd(&c->bar_gen, 1u);
+      vc->t_first = ~0ULL;
+      grid_release(&c->bar_gen, target);
     } else {
-      u32 ns = 32;
-      while (ld_acquire_u32(&c->bar_gen) == gen) {
-        __nanosleep(ns);
-        if (ns < 128) ns <<= 1;
-      }
+      grid_wait(&c->bar_gen, target);
     }
-    __threadfence();
     volatile Ctl* vc = c;
     sm.mode = vc->mode;
     sm.cur = vc->cur;
@@ -1118,7 +1174,8 @@ __device__ void phase1(const Params& p, Smem& sm) {
   u32 owed = 0;  // thread 0: completions of claimed entries held back while the CTA chases locally
   if (threadIdx.x == 0) {
     sm.loc_on = (!ABL && (p.claim_max & LOCAL_CHASE)) ? 1u : 0u;
-    sm.loc_lim = min((p.claim_max >> LOCAL_LIM_SHIFT) & 1023u, LOC_CAP);
+    // >= 1: a zero limit would leave loc_n growing while nothing drains it (pend never 0)
+    sm.loc_lim = max(1u, min((p.claim_max >> LOCAL_LIM_SHIFT) & LOCAL_LIM_MASK, LOC_CAP));
   }
   for (;;) {
     if (threadIdx.x == 0) {
@@ -1169,6 +1226,24 @@ __device__ void phase1(const Params& p, Smem& sm) {
       sm.claim_h = h;
       sm.claim_src = loc;
       sm.st[ST_P_CLAIM] += (unsigned long long)(clock64() - t_c);
+      if (blockIdx.x % SAMPLE_EVERY == 0) {  // claim timeline (which = 100): tail / pend / ticket
+        const u32 k = atomicAdd(&p.ctl->sample_n, 1u);
+        if (k < SAMPLE_CAP) {
+          const u64 wv = ld_relaxed_u64(&sc->word);
+          TraceEnt e;
+          e.t_ns = globaltimer();
+          e.which = 100;
+          e.cur = sm.cur;
+          e.tail = (u32)(wv >> 32);
+          e.mode = n;
+          e.far_min = (u32)wv;
+          e.pad = h;
+          e.closed_b = blockIdx.x;
+          e.closed_c = loc;
+          e.t_first = e.t_rel = 0;
+          p.trace[TRACE_CAP + k] = e;
+        }
+      }
     }
     __syncthreads();
     const u32 n = sm.claim_n;
@@ -1381,7 +1456,7 @@ __device__ void p2_compact(const Params& p, Smem& sm) {
   }
   st_add(sm, ST_HEAVYV, c_live);
   st_add(sm, ST_HEAVY, c_arcs);
-  if (p.flags & 24u) {
+  {
     const u32 cs = __reduce_add_sync(SSSP_FULL_MASK, c_live);
     if (lane == 0 && cs) atomicAdd(&p.ctl->csum, cs);
   }
@@ -1506,6 +1581,57 @@ __device__ void p2_relax(const Params& p, Smem& sm) {
 // most vertices find a hub of the bucket among their lightest heavy arcs and
 // stop early. Every heavy arc out of bucket cur that could improve v is still
 // examined, so the result is the one push-style phase 2 gives.
+// Bucket cur's bounds for the pull: u32 [lo, hi) (INF = 0xFFFFFFFF is never inside, even when
+// hi > 2^32 - 1); f32 by bucket_of, with lo_f <= every distance of bucket cur (cur * Delta
+// rounded down, less 2^-20 relative), so fl(lo_f + w) bounds fl(du + w) from below for every u
+// of the bucket (fl is monotone). f32 graphs carry Delta's bits in delta_u when pulling.
+struct PullBounds {
+  u64 lo, hi;
+  float lo_f;
+  u32 cur;
+};
+template <bool F32>
+__device__ __forceinline__ PullBounds pull_bounds(const Params& p, u32 cur) {
+  PullBounds b;
+  b.cur = cur;
+  b.lo = F32 ? 0 : (u64)cur * p.delta_u;
+  b.hi = F32 ? 0 : b.lo + p.delta_u;
+  b.lo_f = (F32 && cur) ? __fmul_rd(__fmul_rd((float)cur, __uint_as_float(p.delta_u)), 0.99999905f) : 0.f;
+  return b;
+}
+template <bool F32>
+__device__ __forceinline__ bool in_bucket(const Params& p, const PullBounds& b, u32 d) {
+  if (F32) return bucket_of<true>(p, d) == b.cur;
+  return d != NONE && (u64)d >= b.lo && (u64)d < b.hi;
+}
+template <bool F32>
+__device__ __forceinline__ bool unsettled(const Params& p, const PullBounds& b, u32 d) {
+  if (F32) return bucket_of<true>(p, d) > b.cur;
+  return d == NONE || (u64)d >= b.hi;
+}
+// A heavy arc of weight w can still beat best (ascending w: once false, false for the rest).
+// An unreached v (best = INF) scans on even when lo + w >= INF, so an overflow is reported.
+template <bool F32>
+__device__ __forceinline__ bool may_win(const PullBounds& b, u32 w, u32 best) {
+  if (F32) return __float_as_uint(__fadd_rn(b.lo_f, __uint_as_float(w))) < best;
+  return b.lo + w < (u64)best || best == NONE;
+}
+// Candidate through u (du in bucket cur) over an arc of weight w: best = min(best, du + w).
+template <bool F32>
+__device__ __forceinline__ void pull_take(u32 du, u32 w, u32& best, bool& of) {
+  if (F32) {
+    best = min(best, __float_as_uint(__fadd_rn(__uint_as_float(du), __uint_as_float(w))));
+  } else {
+    const u64 cand = (u64)du + w;
+    if (cand >= (u64)NONE)
+      of = true;  // same rule as the push relaxation (relax_finish)
+    else if (cand < (u64)best)
+      best = (u32)cand;
+  }
+}
+
+constexpr u32 PULL_LANE_STEPS = 4;  // a lane scans <= 4 * 2 heavy arcs of a vertex, then hands it off
+
 template <bool F32, bool PRO>
 __device__ void pull_phase(const Params& p, Smem& sm) {
   const u32 cur = sm.cur, lim = sm.lim, lane = lane_id();
@@ -1515,76 +1641,210 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
          i += (i64)gridDim.x * blockDim.x)
       st_relaxed_u64(q + i, SENTINEL);
   }
-  // u32: bucket cur = [lo, hi). f32 (delta_u holds Delta's bits): membership by bucket_of, and
-  // lo_f <= every distance of bucket cur (cur * Delta rounded down, less 2^-20 relative), so
-  // fl(lo_f + w) is a lower bound of fl(du + w) for every u of the bucket (fl is monotone).
-  const u64 lo = F32 ? 0 : (u64)cur * p.delta_u, hi = F32 ? 0 : lo + p.delta_u;
-  const float lo_f = (F32 && cur) ? __fmul_rd(__fmul_rd((float)cur, __uint_as_float(p.delta_u)), 0.99999905f) : 0.f;
-  u32 c_pull = 0, c_arcs = 0;
+  const PullBounds B = pull_bounds<F32>(p, cur);
+  // Candidates: every vertex (first pull), else the list the previous pull kept -- the vertices
+  // that were unsettled then and have arcs (a vertex settled since is skipped, one settled in
+  // bucket cur is counted in C_i). This pull keeps the ones still unsettled after bucket cur.
+  const u32 sel = sm.pull_sel, osel = sel == 0 ? 1u : 0u;
+  const u32* in = sel == 2 ? nullptr : p.xd + (u64)(1 + sel) * p.V;
+  const u32 n_in = sm.pull_n_in;  // first pull: [0, first_n)
+  u32* out = p.xd + (u64)(1 + osel) * p.V;
+  u32* out_n = &p.ctl->pull_n[osel];
+  uint4* longq = reinterpret_cast<uint4*>(p.xd + ((3 * (u64)p.V + 3) & ~3ULL));  // 16-B aligned
+  const u32 long_cap = p.V / 2;
+  constexpr int NV = UNROLL;  // candidates per lane in flight (stage_pushes takes UNROLL)
+  constexpr int PU = 2;       // heavy arcs per candidate per step
+  u32 c_pull = 0, c_arcs = 0, c_in = 0;
+  bool of = false;
   const u64 pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
-  const i64 nt = (i64)gridDim.x * blockDim.x;
-  for (i64 b = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL; b < p.V; b += nt) {
-    const i64 v = b + lane;
-    u32 dv = 0, j = 0, e = 0;
-    bool act = v < p.V;
-    if (act) {
-      dv = ld_cg(p.dist + v);
-      act = F32 ? bucket_of<true>(p, dv) > cur : (u64)dv >= hi;
-    }
-    if (act) {
-      const uint2 r = p.rowc[v];
-      j = PRO ? r.y : r.x;
-      e = p.rowc[v + 1].x;
-      act = j < e;
-    }
-    u32 best = dv;
-    while (__any_sync(SSSP_FULL_MASK, act)) {
-      uint2 a[UNROLL];
-      u32 du[UNROLL];
-      bool ok[UNROLL];
+  const u64 wstride = (u64)gridDim.x * blockDim.x * NV;
+  for (u64 wb = ((u64)blockIdx.x * blockDim.x + (threadIdx.x & ~31u)) * NV; wb < n_in; wb += wstride) {
+    u32 v[NV], dv[NV], j[NV], e[NV], best[NV];
+    bool act[NV], keep[NV];
 #pragma unroll
-      for (int k = 0; k < UNROLL; ++k) a[k] = ld_arc(p.arcs + j + k, act && j + k < e, pol_stream);
+    for (int k = 0; k < NV; ++k) {
+      const u64 i = wb + (u64)k * 32 + lane;
+      v[k] = i < n_in ? (in ? ld_cg(in + i) : (u32)i) : NONE;
+    }
 #pragma unroll
-      for (int k = 0; k < UNROLL; ++k) {
-        ok[k] = act && j + k < e &&  // ascending w: once the bound fails, later arcs cannot win
-                (F32 ? __float_as_uint(__fadd_rn(lo_f, __uint_as_float(a[k].y))) < best : lo + a[k].y < (u64)best);
-        if (!PRO) ok[k] = ok[k] && a[k].y >= p.delta_bits;  // heavy arcs only
-        du[k] = ld_probe(p.dist + a[k].x, ok[k], pol_keep);
+    for (int k = 0; k < NV; ++k) dv[k] = v[k] != NONE ? ld_cg(p.dist + v[k]) : 0u;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      const bool has = v[k] != NONE;
+      c_in += has && in_bucket<F32>(p, B, dv[k]);
+      act[k] = has && unsettled<F32>(p, B, dv[k]);
+      j[k] = e[k] = 0;
+    }
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      if (act[k]) {
+        const uint2 r = p.rowc[v[k]];
+        e[k] = p.rowc[v[k] + 1].x;
+        keep[k] = e[k] > r.x;  // isolated vertices are never reached: drop them
+        j[k] = PRO ? r.y : r.x;
+      } else {
+        keep[k] = false;
       }
+      act[k] = act[k] && j[k] < e[k];
+      best[k] = dv[k];
+    }
+    {  // the next pull's candidates: one reservation per warp
+      u32 m[NV], tot = 0;
 #pragma unroll
-      for (int k = 0; k < UNROLL; ++k) {
-        if constexpr (F32) {
-          if (ok[k] && bucket_of<true>(p, du[k]) == cur) {  // u settled in bucket cur
-            const u32 cand = __float_as_uint(__fadd_rn(__uint_as_float(du[k]), __uint_as_float(a[k].y)));
-            best = min(best, cand);
-          }
-        } else {
-          if (ok[k] && (u64)du[k] >= lo && (u64)du[k] < hi) {  // u settled in bucket cur
-            const u64 cand = (u64)du[k] + a[k].y;
-            if (cand < (u64)best) best = (u32)min(cand, (u64)NONE);
-          }
+      for (int k = 0; k < NV; ++k) {
+        m[k] = __ballot_sync(SSSP_FULL_MASK, keep[k]);
+        tot += __popc(m[k]);
+      }
+      u32 base = 0;
+      if (lane == 0 && tot) base = atomicAdd(out_n, tot);
+      base = __shfl_sync(SSSP_FULL_MASK, base, 0);
+      const u32 lt = lanemask_lt();
+#pragma unroll
+      for (int k = 0; k < NV; ++k) {
+        if (keep[k]) out[base + __popc(m[k] & lt)] = v[k];
+        base += __popc(m[k]);
+      }
+    }
+    bool any = false;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) any |= act[k];
+    u32 steps = 0;
+    while (__any_sync(SSSP_FULL_MASK, any)) {
+      if (steps == PULL_LANE_STEPS) {  // long scans: hand them to whole warps (MODE_PULL_LONG)
+        u32 m[NV], tot = 0;
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+          m[k] = __ballot_sync(SSSP_FULL_MASK, act[k]);
+          tot += __popc(m[k]);
         }
+        u32 base = 0;
+        if (lane == 0) base = atomicAdd(&p.ctl->long_n, tot);
+        base = __shfl_sync(SSSP_FULL_MASK, base, 0);
+        const u32 lt = lanemask_lt();
+        any = false;
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+          const u32 idx = base + __popc(m[k] & lt);
+          if (act[k] && idx < long_cap) {
+            longq[idx] = make_uint4(v[k], j[k], best[k], dv[k]);
+            act[k] = false;
+            v[k] = NONE;  // its push is the long step's
+          }
+          base += __popc(m[k]);
+          any |= act[k];
+        }
+        if (lane == 0 && base > long_cap) atomicMin(&p.ctl->long_n, long_cap);  // the rest stay here
+        if (!__any_sync(SSSP_FULL_MASK, any)) break;
       }
-      if (act) c_arcs += min((u32)UNROLL, e - j);
-      j += UNROLL;
-      act = act && j < e && (PRO ? ok[UNROLL - 1] : true);
+      ++steps;
+      uint2 a[NV][PU];
+#pragma unroll
+      for (int k = 0; k < NV; ++k)
+#pragma unroll
+        for (int u = 0; u < PU; ++u) a[k][u] = ld_arc(p.arcs + j[k] + u, act[k] && j[k] + u < e[k], pol_stream);
+      u32 du[NV][PU];
+      bool ok[NV][PU];
+#pragma unroll
+      for (int k = 0; k < NV; ++k)
+#pragma unroll
+        for (int u = 0; u < PU; ++u) {
+          bool o = act[k] && j[k] + u < e[k] && may_win<F32>(B, a[k][u].y, best[k]);
+          if (!PRO) o = o && a[k][u].y >= p.delta_bits;  // heavy arcs only
+          ok[k][u] = o;
+          du[k][u] = ld_probe(p.dist + a[k][u].x, o, pol_keep);
+        }
+      any = false;
+#pragma unroll
+      for (int k = 0; k < NV; ++k) {
+#pragma unroll
+        for (int u = 0; u < PU; ++u)
+          if (ok[k][u] && in_bucket<F32>(p, B, du[k][u])) pull_take<F32>(du[k][u], a[k][u].y, best[k], of);
+        if (act[k]) c_arcs += min((u32)PU, e[k] - j[k]);
+        j[k] += PU;
+        act[k] = act[k] && j[k] < e[k] && (PRO ? ok[k][PU - 1] : true);
+        any |= act[k];
+      }
     }
+    bool want[UNROLL];
+    u32 nd[UNROLL];
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      want[k] = v[k] != NONE && best[k] < dv[k];
+      nd[k] = best[k];
+      if (want[k]) {
+        atomicMin(p.dist + v[k], best[k]);  // v is this thread's alone during the pull
+        ++c_pull;
+      }
+    }
+    stage_pushes<F32>(p, sm, lim, NONE, want, v, nd);
+  }
+  if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
+  if (!F32 && of) atomicOr(&p.ctl->err, ERR_OVERFLOW);
+  st_add(sm, ST_HEAVY, c_arcs);
+  st_add(sm, ST_HEAVYV, c_pull);
+  {
+    const u32 cs = __reduce_add_sync(SSSP_FULL_MASK, c_in);
+    if (lane == 0 && cs) atomicAdd(&p.ctl->csum, cs);
+  }
+}
+
+// Second step of the pull: the vertices whose weight-sorted heavy scan outlasted the lane
+// budget, one warp per vertex, 64 arcs per step (two per lane), warp-min of the candidates;
+// the scan ends at the first arc that can no longer win (or the segment end).
+template <bool F32, bool PRO>
+__device__ void pull_long(const Params& p, Smem& sm) {
+  const u32 cur = sm.cur, lim = sm.lim, lane = lane_id();
+  const PullBounds B = pull_bounds<F32>(p, cur);
+  const uint4* longq = reinterpret_cast<const uint4*>(p.xd + ((3 * (u64)p.V + 3) & ~3ULL));
+  const u32 n = ld_relaxed_u32(&p.ctl->long_n);
+  const u64 pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
+  u32 c_pull = 0, c_arcs = 0;
+  bool of = false;
+  for (;;) {
+    u32 i = 0;
+    if (lane == 0) i = atomicAdd(&p.ctl->long_head, 1u);
+    i = __shfl_sync(SSSP_FULL_MASK, i, 0);
     bool want[UNROLL] = {};
     u32 vv[UNROLL] = {}, nd[UNROLL] = {};
-    if (v < p.V && best < dv) {
-      if (!F32 && best >= NONE) {
-        atomicOr(&p.ctl->err, ERR_OVERFLOW);
-      } else {
+    if (i < n) {
+      const uint4 it = __ldcg(longq + i);
+      const u32 v = it.x, e = p.rowc[v + 1].x, dv = it.w;
+      u32 j = it.y, best = it.z;
+      for (;;) {
+        uint2 a[2];
+        bool ok[2];
+        u32 du[2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) a[u] = ld_arc(p.arcs + j + u * 32 + lane, j + u * 32 + lane < e, pol_stream);
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          ok[u] = j + u * 32 + lane < e && may_win<F32>(B, a[u].y, best);
+          if (!PRO) ok[u] = ok[u] && a[u].y >= p.delta_bits;
+          du[u] = ld_probe(p.dist + a[u].x, ok[u], pol_keep);
+        }
+        u32 b = best;
+#pragma unroll
+        for (int u = 0; u < 2; ++u)
+          if (ok[u] && in_bucket<F32>(p, B, du[u])) pull_take<F32>(du[u], a[u].y, b, of);
+        best = __reduce_min_sync(SSSP_FULL_MASK, b);
+        if (lane == 0) c_arcs += min(64u, e - j);
+        j += 64;
+        // an arc that failed the bound (or the segment end) ends the scan: weights ascend
+        if (!__all_sync(SSSP_FULL_MASK, ok[0] && ok[1]) || j >= e) break;
+      }
+      if (lane == 0 && best < dv) {
         atomicMin(p.dist + v, best);
         want[0] = true;
-        vv[0] = (u32)v;
+        vv[0] = v;
         nd[0] = best;
         ++c_pull;
       }
     }
     stage_pushes<F32>(p, sm, lim, NONE, want, vv, nd);
+    if (i >= n) break;
   }
   if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
+  if (!F32 && of) atomicOr(&p.ctl->err, ERR_OVERFLOW);
   st_add(sm, ST_HEAVY, c_arcs);
   st_add(sm, ST_HEAVYV, c_pull);
 }
@@ -1703,7 +1963,8 @@ template <bool F32, bool PRO, bool ABL>
 __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) {
   __shared__ Smem sm;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
-    TraceEnt e = {globaltimer(), 99u, 0u, 0u, 0u, 0u, 0u};
+    const u64 t0 = globaltimer();
+    TraceEnt e = {t0, 99u, 0u, 0u, 0u, 0u, 0u, NONE, 0u, t0, t0};
     p.trace[0] = e;
     p.ctl->trace_n = 1;
   }
@@ -1734,6 +1995,9 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
       grid_barrier(p, sm, SYNC_P2);
     } else if (mode == MODE_PULL) {
       pull_phase<F32, PRO>(p, sm);
+      grid_barrier(p, sm, SYNC_PL);
+    } else if (mode == MODE_PULL_LONG) {
+      pull_long<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
     } else if (ABL && mode == MODE_MERGE) {  // extended build only (adaptive Delta)
       if constexpr (ABL) merge_slots<F32>(p, sm);
@@ -1760,6 +2024,12 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
   }
   __syncthreads();
   if (threadIdx.x < ST_N && sm.st[threadIdx.x]) atomicAdd(p.stats + threadIdx.x, sm.st[threadIdx.x]);
+  // Every CTA has passed the last grid barrier, so err is final: fold it into the sticky word
+  // that sssp_wait / sssp_run_batch / sssp_distances report (and clear) on the host.
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const u32 e = ld_relaxed_u32(&p.ctl->err);
+    if (e) atomicOr(&p.ctl->err_acc, e);
+  }
 }
 
 // ------------------------------------------------------------- init -------
@@ -1774,6 +2044,7 @@ struct AdaptInit {
   u32 mode;        // 0 fixed Delta, 1 / 2 adaptive (readings A / B of Eq. (2))
   float d0;        // Delta_0 in fine units
   u32 m0, mmin, mmax, lvl0;
+  u32 first_n;     // ids [0, first_n) hold every vertex with arcs and the source
 };
 __global__ void k_seed(Params p, u32 src, AdaptInit ai) {
   const u32 t = threadIdx.x;
@@ -1796,6 +2067,8 @@ __global__ void k_seed(Params p, u32 src, AdaptInit ai) {
     c->p2_begin = c->p2_end = c->p2_head = 0;
     c->err = 0;
     c->bar_count = 0;
+    c->bar_gen = 0;
+    c->t_first = ~0ULL;
     c->epochs = 1;
     c->rescans = 0;
     c->rescan_base = 0;
@@ -1818,6 +2091,13 @@ __global__ void k_seed(Params p, u32 src, AdaptInit ai) {
     c->a_m = ai.m0;
     c->lvl = ai.lvl0;
     c->csum = 0;
+    c->pull_sel = 2;  // the first pull scans every vertex
+    c->pull_n[0] = c->pull_n[1] = 0;
+    c->closed_b = NONE;
+    c->closed_c = 0;
+    c->long_n = c->long_head = 0;
+    c->sample_n = 0;
+    c->first_n = ai.first_n;
   }
 }
 

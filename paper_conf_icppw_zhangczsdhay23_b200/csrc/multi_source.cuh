@@ -501,23 +501,13 @@ __device__ void ms_grid_barrier(const MParams& p, MSmem& sm) {
   __syncthreads();
   if (threadIdx.x == 0) {
     MCtl* c = p.ctl;
-    const u32 gen = ld_acquire_u32(&c->bar_gen);
-    __threadfence();
-    const u32 arrived = atomicAdd(&c->bar_count, 1u);
-    if (arrived == gridDim.x - 1) {
-      c->bar_count = 0;
-      __threadfence();
+    u32 target;
+    if (grid_arrive(&c->bar_count, &target)) {
       ms_decide(p);
-      __threadfence();
-      atomicAdd(&c->bar_gen, 1u);
+      grid_release(&c->bar_gen, target);
     } else {
-      u32 ns = 32;
-      while (ld_acquire_u32(&c->bar_gen) == gen) {
-        __nanosleep(ns);
-        if (ns < 128) ns <<= 1;
-      }
+      grid_wait(&c->bar_gen, target);
     }
-    __threadfence();
     volatile MCtl* vc = c;
     sm.mode = vc->mode;
     sm.cur = vc->cur;
@@ -631,6 +621,7 @@ __global__ void k_ms_seed(MParams p, const u32* __restrict__ src, u32 n) {
   c->rescans = 0;
   c->base = 0;
   c->bar_count = 0;
+  c->bar_gen = 0;
 }
 
 // out[l * ld + o] = D[old2new[o]][l] for l < n (a8 for the group; f32 bits as is).

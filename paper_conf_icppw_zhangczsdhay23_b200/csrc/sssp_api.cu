@@ -99,6 +99,8 @@ struct sssp_graph_s {
   // params
   i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP;
   i64 hub_ids_cached = -1;
+  int sym_state = -1;  // arc multiset symmetric? -1 unknown (checked on demand after a weight sort)
+  i64 v_nz = -1;       // degree-sorted graphs: vertices with arcs are ids [0, v_nz); -1 unknown
   i64 l2_window_bytes = -1;  // -1: not configured yet
   float l2_hit_ratio = 1.f;
 };
@@ -184,10 +186,10 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
     CG(cudaMalloc(&g->rowc, sizeof(uint2) * (V + 1)));
     CG(cudaMalloc(&g->arcs, sizeof(uint2) * std::max<i64>(A, 1)));
     CG(cudaMalloc(&g->dist, sizeof(u32) * V));
-    CG(cudaMalloc(&g->xd, sizeof(u32) * V));
+    CG(cudaMalloc(&g->xd, sizeof(u32) * (5 * V + 4)));  // sweep marks, two pull candidate lists, long scans
     CG(cudaMalloc(&g->ctl, sizeof(Ctl)));
     CG(cudaMalloc(&g->stats, sizeof(unsigned long long) * ST_N));
-    CG(cudaMalloc(&g->trace, sizeof(TraceEnt) * TRACE_CAP));
+    CG(cudaMalloc(&g->trace, sizeof(TraceEnt) * (TRACE_CAP + SAMPLE_CAP)));
     CG(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
     CG(cudaMemsetAsync(g->stats, 0, sizeof(unsigned long long) * ST_N, s));
     for (int i = 0; i < 4; ++i) CG(cudaEventCreate(&g->ev[i]));
@@ -334,6 +336,11 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       return SSSP_OK;
     case SSSP_PARAM_PULL_SYMMETRIC:
       if (v != 0 && v != 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "pull is 0 or 1");
+      if (v && (g->pro_flags & SSSP_PRO_WEIGHT)) {  // layout ready: verify the assertion now
+        int sym = 0;
+        if ((s = sssp_is_symmetric(g, &sym))) return s;
+        if (!sym) return fail(SSSP_ERR_INVALID_STATE, "pull phases need a symmetric graph; this one is not");
+      }
       g->p_pull = v;
       return SSSP_OK;
     case SSSP_PARAM_LOCAL_CHASE:
@@ -350,6 +357,34 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       return SSSP_OK;
   }
   return fail(SSSP_ERR_INVALID_ARGUMENT, "unknown parameter %d", (int)p);
+}
+
+// ------------------------------------------------------------- symmetry --
+extern "C" sssp_status sssp_is_symmetric(sssp_graph_t g, int* out) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+  if (!(g->pro_flags & SSSP_PRO_WEIGHT))
+    return fail(SSSP_ERR_INVALID_STATE, "the symmetry check needs weight-sorted adjacencies (sssp_reorder)");
+  if (g->sym_state < 0) {
+    DeviceGuard dg(g->device);
+    cudaStream_t s = g->stream;
+    u32* flag = nullptr;
+    u32 h = 0;
+    CU(cudaMallocAsync(&flag, sizeof(u32), s));
+    CU(cudaMemsetAsync(flag, 0, sizeof(u32), s));
+    if (g->A > 0) {
+      const i64 nb = std::min<i64>((g->A + SYM_PER_BLOCK - 1) / SYM_PER_BLOCK, (i64)g->num_sms * 16);
+      k_check_symmetric<<<(unsigned)nb, 256, 0, s>>>(g->rowp, g->arcs, g->V, g->A, flag);
+      CU(cudaGetLastError());
+    }
+    CU(cudaMemcpyAsync(&h, flag, sizeof(u32), cudaMemcpyDeviceToHost, s));
+    CU(cudaFreeAsync(flag, s));
+    CU(cudaStreamSynchronize(s));
+    g->sym_state = h ? 0 : 1;
+  }
+  *out = g->sym_state;
+  return SSSP_OK;
 }
 
 // --------------------------------------------------------------- reorder --
@@ -389,58 +424,91 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   cudaStream_t s = g->stream;
   const i64 V = g->V, A = g->A;
   const bool deg = flags & SSSP_PRO_DEGREE, wsort = flags & SSSP_PRO_WEIGHT;
-  CU(cudaEventRecord(g->ev[2], s));
-  // temporaries
+  // Every temporary is allocated before the timed window and freed after it, with
+  // plain cudaMalloc (one-off, ~24 B per arc: not worth keeping in a stream pool),
+  // and no host round trip happens inside the window: reorder_ms is device time.
   const i64 nmax = std::max<i64>(std::max(V, A), 1);
   const i64 ntiles_max = (nmax + RS_TILE - 1) / RS_TILE;
   const i64 hist_n = 256 * ntiles_max;
-  u32 *hist = nullptr, *tmp = nullptr, *f[6] = {}, *dmax = nullptr;
+  const u32 nh_cap = (u32)(A / EXPAND_HUB + 1);
+  std::vector<void*> temps;
+  auto alloc = [&](void** ptr, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMalloc(ptr, std::max<size_t>(bytes, 4));
+    if (e == cudaSuccess) temps.push_back(*ptr);
+    return e;
+  };
+  auto free_all = [&]() {
+    for (void* t : temps) cudaFree(t);
+    temps.clear();
+  };
+  u32 *hist = nullptr, *tmp = nullptr, *f[6] = {}, *dmax = nullptr, *key0 = nullptr, *key1 = nullptr,
+      *id1 = nullptr, *hubs = nullptr, *cst = nullptr, *ctmp = nullptr;
   u64 *ndeg = nullptr, *stmp = nullptr;
-  CU(cudaMallocAsync(&hist, sizeof(u32) * hist_n, s));
-  CU(cudaMallocAsync(&tmp, sizeof(u32) * scan_tmp_elems(hist_n), s));
-  CU(cudaMallocAsync(&dmax, sizeof(u32), s));
-  CU(cudaMemsetAsync(dmax, 0, sizeof(u32), s));
+  {
+    cudaError_t e = cudaSuccess;
+    auto A_ = [&](cudaError_t x) {
+      if (e == cudaSuccess) e = x;
+    };
+    A_(alloc((void**)&hist, sizeof(u32) * hist_n));
+    A_(alloc((void**)&tmp, sizeof(u32) * scan_tmp_elems(hist_n)));
+    A_(alloc((void**)&dmax, sizeof(u32)));
+    if (deg) {
+      if (!g->new2old) A_(cudaMalloc(&g->new2old, sizeof(u32) * V));
+      if (!g->old2new) A_(cudaMalloc(&g->old2new, sizeof(u32) * V));
+      A_(alloc((void**)&key0, sizeof(u32) * V));
+      A_(alloc((void**)&key1, sizeof(u32) * V));
+      A_(alloc((void**)&id1, sizeof(u32) * V));
+      A_(alloc((void**)&ndeg, sizeof(u64) * (V + 1)));
+      A_(alloc((void**)&stmp, sizeof(u64) * scan_tmp_elems(V)));
+    }
+    if (A > 0) {
+      for (int i = 0; i < 6; ++i) A_(alloc((void**)&f[i], sizeof(u32) * A));
+      A_(alloc((void**)&hubs, sizeof(u32) * (nh_cap + 1)));
+      A_(alloc((void**)&cst, sizeof(u32) * (nh_cap + 1)));
+      A_(alloc((void**)&ctmp, sizeof(u32) * scan_tmp_elems(nh_cap + 1)));
+    }
+    if (e != cudaSuccess) {
+      free_all();
+      cudaGetLastError();
+      return fail(e == cudaErrorMemoryAllocation ? SSSP_ERR_OUT_OF_MEMORY : SSSP_ERR_CUDA,
+                  "reorder temporaries: %s", cudaGetErrorString(e));
+    }
+  }
+#define CT(call)                \
+  do {                          \
+    cudaError_t e_ = (call);    \
+    if (e_ != cudaSuccess) {    \
+      free_all();               \
+      g->sticky_cuda = true;    \
+      return fail(SSSP_ERR_CUDA, "reorder: %s: %s", #call, cudaGetErrorString(e_)); \
+    }                           \
+  } while (0)
+  CT(cudaMemsetAsync(dmax, 0, sizeof(u32), s));
+  CT(cudaEventRecord(g->ev[2], s));
   if (deg) {
-    // a1: stable radix sort of (maxdeg - deg, id) -> new2old (desc degree, asc id)
-    if (!g->new2old) CU(cudaMalloc(&g->new2old, sizeof(u32) * V));
-    if (!g->old2new) CU(cudaMalloc(&g->old2new, sizeof(u32) * V));
-    u32 *key0, *key1, *id1;
-    CU(cudaMallocAsync(&key0, sizeof(u32) * V, s));
-    CU(cudaMallocAsync(&key1, sizeof(u32) * V, s));
-    CU(cudaMallocAsync(&id1, sizeof(u32) * V, s));
+    // a1: stable radix sort of (maxdeg - deg, id) -> new2old (desc degree, asc id). maxdeg <= A,
+    // so bits_for(A) passes cover it without reading maxdeg back to the host.
     k_max_degree<<<grid_for(V), 256, 0, s>>>(g->rowp, V, dmax);
     k_degree_keys<<<grid_for(V), 256, 0, s>>>(g->rowp, V, dmax, key0, g->new2old);
-    u32 maxdeg = 0;
-    CU(cudaMemcpyAsync(&maxdeg, dmax, sizeof(u32), cudaMemcpyDeviceToHost, s));
-    CU(cudaStreamSynchronize(s));
     Fields<2> a{{key0, g->new2old}}, b{{key1, id1}};
-    const int nb = bits_for(maxdeg);
+    const int nb = std::max(1, bits_for((u64)A));
     for (int sh = 0; sh < nb; sh += 8) {
-      st = radix_pass<2>(g, a, b, 0, V, sh, hist, tmp);
-      if (st) return st;
+      if ((st = radix_pass<2>(g, a, b, 0, V, sh, hist, tmp))) {
+        free_all();
+        return st;
+      }
     }
-    if (a.f[1] != g->new2old) CU(cudaMemcpyAsync(g->new2old, a.f[1], sizeof(u32) * V, cudaMemcpyDeviceToDevice, s));
-    CU(cudaMallocAsync(&ndeg, sizeof(u64) * (V + 1), s));
-    CU(cudaMallocAsync(&stmp, sizeof(u64) * scan_tmp_elems(V), s));
+    if (a.f[1] != g->new2old) CT(cudaMemcpyAsync(g->new2old, a.f[1], sizeof(u32) * V, cudaMemcpyDeviceToDevice, s));
     k_invert_perm<<<grid_for(V), 256, 0, s>>>(g->new2old, g->rowp, V, g->old2new, ndeg);
     scan_exclusive_rec<u64>(ndeg, ndeg, V, stmp, s);  // new row starts
-    CU(cudaFreeAsync(key0, s));
-    CU(cudaFreeAsync(key1, s));
-    CU(cudaFreeAsync(id1, s));
-    CU(cudaGetLastError());
+    CT(cudaGetLastError());
   }
   if (A > 0) {
     // a2+a3: one stable LSD radix sort of all arcs by (new src, w, new dst)
-    for (int i = 0; i < 6; ++i) CU(cudaMallocAsync(&f[i], sizeof(u32) * A, s));
     // arcs of vertices with <= EXPAND_HUB arcs: warp-flattened; hubs: 4096-arc
     // chunks over all blocks. The hub count is bounded by A / EXPAND_HUB, so
     // the chunk scan runs over that capacity with no host round trip.
-    const u32 nh_cap = (u32)(A / EXPAND_HUB + 1);
-    u32 *hubs = nullptr, *cst = nullptr, *ctmp = nullptr;
-    CU(cudaMallocAsync(&hubs, sizeof(u32) * (nh_cap + 1), s));
-    CU(cudaMallocAsync(&cst, sizeof(u32) * (nh_cap + 1), s));
-    CU(cudaMallocAsync(&ctmp, sizeof(u32) * scan_tmp_elems(nh_cap + 1), s));
-    CU(cudaMemsetAsync(hubs + nh_cap, 0, sizeof(u32), s));
+    CT(cudaMemsetAsync(hubs + nh_cap, 0, sizeof(u32), s));
     k_list_hubs<<<grid_for(V), 256, 0, s>>>(g->rowp, V, hubs, hubs + nh_cap);
     k_expand_arcs_flat<<<grid_for(V), 256, 0, s>>>(g->rowp, g->arcs, V, deg ? g->old2new : nullptr,
                                                    f[0], f[1], f[2]);
@@ -448,47 +516,42 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
     scan_exclusive_rec<u32>(cst, cst, (i64)nh_cap + 1, ctmp, s);
     k_expand_hubs<<<g->num_sms * 8, 256, 0, s>>>(g->rowp, g->arcs, hubs, nh_cap, cst,
                                                  deg ? g->old2new : nullptr, f[0], f[1], f[2]);
-    CU(cudaFreeAsync(hubs, s));
-    CU(cudaFreeAsync(cst, s));
-    CU(cudaFreeAsync(ctmp, s));
-    CU(cudaGetLastError());
+    CT(cudaGetLastError());
     Fields<3> a{{f[0], f[1], f[2]}}, b{{f[3], f[4], f[5]}};
     const int vb = bits_for((u64)(V - 1));
+    auto pass3 = [&](int kf, int sh) { return radix_pass<3>(g, a, b, kf, A, sh, hist, tmp); };
     if (wsort) {
-      for (int sh = 0; sh < vb; sh += 8)
-        if ((st = radix_pass<3>(g, a, b, 2, A, sh, hist, tmp))) return st;
+      for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(2, sh);
       const int wb = bits_for(g->maxw_bits);
-      for (int sh = 0; sh < wb; sh += 8)
-        if ((st = radix_pass<3>(g, a, b, 1, A, sh, hist, tmp))) return st;
+      for (int sh = 0; sh < wb && !st; sh += 8) st = pass3(1, sh);
     }
     if (deg || wsort)
-      for (int sh = 0; sh < vb; sh += 8)
-        if ((st = radix_pass<3>(g, a, b, 0, A, sh, hist, tmp))) return st;
+      for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(0, sh);
+    if (st) {
+      free_all();
+      return st;
+    }
     k_pack_sorted<<<grid_for(A), 256, 0, s>>>(a.f[1], a.f[2], A, g->arcs);
-    CU(cudaGetLastError());
-    for (int i = 0; i < 6; ++i) CU(cudaFreeAsync(f[i], s));
+    CT(cudaGetLastError());
   }
-  if (deg) {
-    k_set_rowp<<<grid_for(V + 1), 256, 0, s>>>(ndeg, V, A, g->rowp);
-    CU(cudaFreeAsync(ndeg, s));
-    CU(cudaFreeAsync(stmp, s));
-  }
-  CU(cudaFreeAsync(hist, s));
-  CU(cudaFreeAsync(tmp, s));
-  CU(cudaFreeAsync(dmax, s));
-  CU(cudaEventRecord(g->ev[3], s));
-  CU(cudaGetLastError());
+  if (deg) k_set_rowp<<<grid_for(V + 1), 256, 0, s>>>(ndeg, V, A, g->rowp);
+  CT(cudaEventRecord(g->ev[3], s));
+  CT(cudaGetLastError());
   if (deg) {
     g->h_old2new.resize(V);
-    CU(cudaMemcpyAsync(g->h_old2new.data(), g->old2new, sizeof(u32) * V, cudaMemcpyDeviceToHost, s));
-    CU(cudaStreamSynchronize(s));
+    CT(cudaMemcpyAsync(g->h_old2new.data(), g->old2new, sizeof(u32) * V, cudaMemcpyDeviceToHost, s));
   }
+  CT(cudaStreamSynchronize(s));
+  free_all();
+#undef CT
   g->pro_flags |= flags;
   g->heavy_valid = false;
   g->rowc_valid = false;
   g->rowc_lv_valid = false;
   g->hubdist_bits = 0xFFFFFFFFu;
   g->hub_ids_cached = -1;
+  g->sym_state = -1;
+  g->v_nz = -1;
   g->have_result = false;
   g->reorder_timed = true;
   return SSSP_OK;
@@ -510,7 +573,7 @@ struct DeltaParams {
 // (u32: max(1, floor(Delta_0 / 4))); a bucket spans m in [Delta_0/4, 4 Delta_0] / g
 // of them (at most 16), and delta_u / inv / delta_bits describe g instead of Delta.
 static void adapt_params(sssp_graph_t g, int mode, DeltaParams* dp) {
-  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
+  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u, 0u};
   if (!mode || dp->delta_bits == 0xFFFFFFFFu || (g->wtype == SSSP_WEIGHT_F32 && dp->inv == 0.f)) return;
   double d0;
   if (g->wtype == SSSP_WEIGHT_U32) {
@@ -532,11 +595,11 @@ static void adapt_params(sssp_graph_t g, int mode, DeltaParams* dp) {
   const u32 m0 = std::min(std::max((u32)std::lrint(d0), mmin), mmax);
   u32 l = 0;
   while ((1u << l) < m0) ++l;
-  dp->ai = AdaptInit{(u32)mode, (float)d0, m0, mmin, mmax, l};
+  dp->ai = AdaptInit{(u32)mode, (float)d0, m0, mmin, mmax, l, 0u};
 }
 
 static sssp_status delta_params(sssp_graph_t g, double delta, DeltaParams* dp) {
-  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
+  dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u, 0u};
   if (std::isnan(delta) || delta <= 0.0) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta must be > 0 (got %g)", delta);
   if (g->wtype == SSSP_WEIGHT_U32) {
     double c = std::ceil(delta);
@@ -701,13 +764,32 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
   if (adapt) p.flags |= (dp.ai.mode == 2 ? 16u : 8u) | (pro ? 64u : 0u);
   if (f32) p.flags |= 32u;
-  if (g->p_pull && pro && !adapt && (f32 ? dp.inv != 0.f : dp.delta_u != 0xFFFFFFFFu)) {  // caller asserted symmetry
+  if (g->p_pull && pro && !adapt && (f32 ? dp.inv != 0.f : dp.delta_u != 0xFFFFFFFFu)) {  // symmetric, checked
+    if (g->sym_state < 0) {
+      int sym = 0;
+      if ((st = sssp_is_symmetric(g, &sym))) return st;
+    }
+    if (g->sym_state == 0) return fail(SSSP_ERR_INVALID_STATE, "pull phases need a symmetric graph; this one is not");
     p.flags |= 128u;
     if (f32) p.delta_u = dp.delta_bits;  // pull_phase needs Delta itself (bucket_of uses inv_delta)
   }
+  // The first pull scans ids [0, first_n): with PRO's degree order the isolated vertices
+  // (never reached, unless the source) are the id tail, found once per reorder.
+  if ((g->pro_flags & SSSP_PRO_DEGREE) && g->v_nz < 0) {
+    u32 lo = 0, hi = (u32)g->V;  // first id with degree 0 (degrees non-increasing)
+    longlong2 r[2];
+    while (lo < hi) {
+      const u32 mid = lo + (hi - lo) / 2;
+      CU(cudaMemcpy(r, g->rowp + mid, 2 * sizeof(longlong2), cudaMemcpyDeviceToHost));
+      if (r[1].x > r[0].x) lo = mid + 1; else hi = mid;
+    }
+    g->v_nz = lo;
+  }
+  AdaptInit ai = dp.ai;
+  ai.first_n = (g->pro_flags & SSSP_PRO_DEGREE) ? (u32)std::max<i64>(g->v_nz, (i64)src_internal + 1) : (u32)g->V;
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
-  k_seed<<<1, 64, 0, s>>>(p, src_internal, dp.ai);
+  k_seed<<<1, 64, 0, s>>>(p, src_internal, ai);
   CU(cudaGetLastError());
   cudaEvent_t e0, e1;
   for (int i = 0; i < 2; ++i) {
@@ -770,15 +852,20 @@ extern "C" sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta) {
 }
 
 // ------------------------------------------------------------ results -----
-static sssp_status check_run_errors(sssp_graph_t g) {
-  Ctl c;
-  CU(cudaMemcpyAsync(&c, g->ctl, sizeof c, cudaMemcpyDeviceToHost, g->stream));
+// Errors of every persistent run since the last report: the kernel ORs its err word into
+// Ctl::err_acc as it exits (k_seed never clears err_acc), so a run whose errors nobody has
+// read yet is never lost. Synchronises the handle's stream, reports, clears.
+static sssp_status take_run_errors(sssp_graph_t g) {
+  u32 e = 0;
+  u32* acc = &g->ctl->err_acc;
+  CU(cudaMemcpyAsync(&e, acc, sizeof e, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaMemsetAsync(acc, 0, sizeof e, g->stream));
   CU(cudaStreamSynchronize(g->stream));
-  if (c.err & ERR_INTERNAL) {
+  if (e & ERR_INTERNAL) {
     g->need_full_reset = true;
     return fail(SSSP_ERR_INTERNAL, "scheduler queue overflow");
   }
-  if (c.err & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
+  if (e & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
   return SSSP_OK;
 }
 
@@ -810,7 +897,7 @@ extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory whe
   k_output<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->old2new, g->V, staged ? g->out_tmp : dst);
   CU(cudaGetLastError());
   if (staged) CU(cudaMemcpyAsync(out, g->out_tmp, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
-  return check_run_errors(g);
+  return take_run_errors(g);
 }
 
 extern "C" sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memory where) {
@@ -858,7 +945,7 @@ extern "C" sssp_status sssp_wait(sssp_graph_t g) {
   DeviceGuard dg(g->device);
   CU(cudaStreamSynchronize(g->stream));
   if (g->d2h) CU(cudaStreamSynchronize(g->d2h));
-  return SSSP_OK;
+  return take_run_errors(g);
 }
 
 extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
@@ -882,7 +969,7 @@ extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, in
     k_output<<<grid_for(g->V), 256, 0, g->stream>>>(g->dist, g->old2new, g->V, (u32*)out_dev + (size_t)i * ld);
     CU(cudaGetLastError());
   }
-  return SSSP_OK;
+  return take_run_errors(g);  // synchronises: errors of any of the n runs
 }
 
 // NEXT-4: up to 32 sources per persistent launch (multi_source.cuh).
@@ -981,15 +1068,21 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
         if (tmp[v + 1].x - tmp[v].x > best) best = tmp[v + 1].x - tmp[v].x, hub = (u32)v;
     }  // degree-sorted (PRO): internal id 0 has the highest degree
     DeltaParams dh = dp;
-    dh.ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u};
+    dh.ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u, 0u};
     g->have_result = false;
+    u32 err_prev = 0;  // errors of earlier, not yet reported sssp_run calls survive this run
+    CU(cudaMemcpyAsync(&err_prev, &g->ctl->err_acc, sizeof(u32), cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
     if ((st = launch_run(g, hub, dh, false))) return st;
     g->h_hubdist.resize(g->V);
     CU(cudaMemcpyAsync(g->h_hubdist.data(), g->dist, sizeof(u32) * g->V, cudaMemcpyDeviceToHost, s));
     CU(cudaStreamSynchronize(s));
+    // the alignment run's own errors are not the batch's (its keys only order the queue)
+    CU(cudaMemcpy(&g->ctl->err_acc, &err_prev, sizeof(u32), cudaMemcpyHostToDevice));
     g->hubdist_bits = dp.delta_bits;
   }
   std::vector<u32> src(2 * MS_LANES, 0u);
+  u32 err_all = 0;
   for (i64 g0 = 0; g0 < n; g0 += MS_LANES) {
     const u32 nn = (u32)std::min<i64>(MS_LANES, n - g0);
     for (u32 l = 0; l < nn; ++l)
@@ -1040,12 +1133,13 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
     CU(cudaEventRecord(e1, s));
     k_ms_output<<<grid_for(g->V), 256, 0, s>>>(g->ms_D, g->old2new, g->V, nn, (u32*)out_dev + (size_t)g0 * ld, ld);
     CU(cudaGetLastError());
+    // k_ms_seed clears err for every group: read this group's before the next one starts
+    u32 e = 0;
+    CU(cudaMemcpyAsync(&e, &g->ms_ctl->err, sizeof e, cudaMemcpyDeviceToHost, s));
     CU(cudaStreamSynchronize(s));  // the source buffer is reused by the next group
+    err_all |= e;
   }
-  MCtl c;
-  CU(cudaMemcpyAsync(&c, g->ms_ctl, sizeof c, cudaMemcpyDeviceToHost, s));
-  CU(cudaStreamSynchronize(s));
-  if (c.err & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
+  if (err_all & ERR_OVERFLOW) return fail(SSSP_ERR_OVERFLOW, "u32 distance overflow");
   return SSSP_OK;
 }
 
@@ -1193,6 +1287,25 @@ extern "C" sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int
   const int64_t k = std::min<int64_t>(n, std::max<int64_t>(max_entries, 0));
   if (k > 0) {
     CU(cudaMemcpyAsync(out, g->trace, sizeof(TraceEnt) * k, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+  }
+  return SSSP_OK;
+}
+
+extern "C" sssp_status sssp_get_samples(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
+                                        int64_t* n_entries) {
+  sssp_status st = check_handle(g);
+  if (st) return st;
+  if (!n_entries || (max_entries > 0 && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad sample buffer");
+  DeviceGuard dg(g->device);
+  Ctl c;
+  CU(cudaMemcpyAsync(&c, g->ctl, sizeof c, cudaMemcpyDeviceToHost, g->stream));
+  CU(cudaStreamSynchronize(g->stream));
+  const int64_t n = std::min<int64_t>(c.sample_n, SAMPLE_CAP);
+  *n_entries = n;
+  const int64_t k = std::min<int64_t>(n, std::max<int64_t>(max_entries, 0));
+  if (k > 0) {
+    CU(cudaMemcpyAsync(out, g->trace + TRACE_CAP, sizeof(TraceEnt) * k, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
   }
   return SSSP_OK;

@@ -429,10 +429,25 @@ def _adapt_records(tr):
     return [e for e in tr if e["which"] == 8]
 
 
+def _closed_buckets(tr):
+    """(first slot, end slot, kernel C) of every bucket the scheduler closed, in order: the
+    closing entry names the bucket (closed_b), its end is the cur_end (pad) that the
+    preceding entries recorded for it."""
+    out, end = [], {}
+    for e in tr:
+        if e["closed_b"] != INF:
+            out.append((e["closed_b"], end[e["closed_b"]], e["closed_c"]))
+        if e["which"] != 8:
+            end[e["cur"]] = e["pad"]
+    return out
+
+
 @pytest.mark.parametrize("mode,reading", [(1, "A"), (2, "B")])
 def test_adaptive_delta_follows_eq1(sssp, mode, reading):
-    """The widths the kernel used are the oracle's Eq. (1)-(2) applied to the
-    kernel's own per-bucket counts C_i (settled) and T_i (phase-1 items)."""
+    """The widths the kernel used are the oracle's Eq. (1)-(2) applied to
+    C_i = vertices whose final distance (oracle Dijkstra) lies in bucket i's
+    recorded bounds -- checked equal to the kernel's own count -- and the
+    kernel's T_i (phase-1 queue items: schedule-dependent)."""
     g = gen.grid(400, 300, p=0.2, seed=8)  # many buckets
     s = int(gen.sample_sources(g, 1, seed=3)[0])
     exp = oracle.dijkstra(g.row, g.col, g.w, s)
@@ -440,10 +455,18 @@ def test_adaptive_delta_follows_eq1(sssp, mode, reading):
         G.reorder()
         G.set_param(sssp.SSSP_PARAM_ADAPTIVE_DELTA, mode)
         assert_same(G.sssp(s, 400), exp, "grid adaptive")
-        recs = _adapt_records(G.trace())
+        tr = G.trace()
+        recs = _adapt_records(tr)
         st = G.stats()
     assert len(recs) >= 20 and st["rescans"] == 0
-    C = [r["cur"] for r in recs]
+    fine = 100  # Delta_0 = 400 = 4 ring slots of g = 100
+    closed = _closed_buckets(tr)
+    assert len(closed) == len(recs) + 1  # the last bucket closes without an Eq. (1) record
+    C = []
+    for i, (r, (b0, b1, kc)) in enumerate(zip(recs, closed)):
+        oc = int(np.count_nonzero((exp != INF) & (exp >= b0 * fine) & (exp < b1 * fine)))
+        assert r["cur"] == kc == oc, f"C_{i}: Eq. (1) record {r['cur']}, trace {kc}, oracle {oc} ([{b0},{b1}))"
+        C.append(oc)
     T = [r["tail"] for r in recs]
     ref = oracle.adaptive_delta(C, T, 4.0, reading)  # Delta_0 = 400 = 4 ring slots of g = 100
     got = [float(np.array([r["far_min"]], dtype=np.uint32).view(np.float32)[0]) for r in recs]
@@ -453,8 +476,45 @@ def test_adaptive_delta_follows_eq1(sssp, mode, reading):
         want = min(max(int(round(b)), 1), 16)
         assert m == want or abs(b - math.floor(b) - 0.5) < 1e-3, f"width {i + 1}: {m} vs {want}"
     assert len(set(r["mode"] for r in recs)) > 1, "Delta never changed"
-    # C_i counts each settled vertex once (the last bucket closes without a record)
-    assert sum(C) <= int((exp != INF).sum())
+    assert sum(c for _, _, c in closed) == int((exp != INF).sum())
+
+
+@pytest.mark.parametrize("case", ["kron-pull", "kron-push", "grid", "kron-noreorder"])
+def test_bucket_settled_counts_match_oracle(sssp, case):
+    """SURVEY §8(c) scheduler stat (ii): for a fixed Delta and u32 weights, the
+    vertices settled in bucket b (trace closed_c) equal #{v : floor(d(v)/Delta) = b}
+    of the oracle's Dijkstra distances (oracle.bucket_histogram; bucket
+    definition), bucket by bucket; every non-empty bucket is closed
+    exactly once and the counts sum to the reachable vertices."""
+    if case == "grid":
+        g, deltas = gen.grid(300, 200, p=0.2, seed=5), (400, 1600, 50)
+    else:
+        g, deltas = gen.kronecker(13, 16, seed=31), (8, 16, 64)
+    srcs = [int(x) for x in gen.sample_sources(g, 2, seed=4)]
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if case != "kron-noreorder":
+            G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1 if case == "kron-pull" else 0)
+        if case == "grid":  # with the local chase on (auto here) the counts are not kept
+            G.sssp(srcs[0], 1600)
+            assert all(e["closed_c"] == INF for e in G.trace() if e["closed_b"] != INF)
+            G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, 0)
+        for s in srcs:
+            exp = oracle.dijkstra(g.row, g.col, g.w, s)
+            for d in deltas:
+                assert_same(G.sssp(s, d), exp, f"{case} delta={d}")
+                closed = [(b, c) for b, _, c in _closed_buckets(G.trace())]
+                hist = oracle.bucket_histogram(exp, d)
+                got = {}
+                for b, c in closed:
+                    assert b not in got, f"bucket {b} closed twice"
+                    got[b] = c
+                for b, c in got.items():
+                    want = int(hist[b]) if b < len(hist) else 0
+                    assert c == want, f"{case} delta={d} src={s} bucket {b}: kernel {c} oracle {want}"
+                nonempty = {b for b in range(len(hist)) if hist[b]}
+                assert nonempty <= set(got), f"buckets never closed: {sorted(nonempty - set(got))[:5]}"
+                assert sum(got.values()) == int((exp != INF).sum())
 
 
 # --------------------------------------- batched multi-source (NEXT-4) ----
@@ -698,3 +758,127 @@ def test_local_chase_parity(sssp):
                             reach = int(np.count_nonzero(e != (INF if g.wtype == "u32" else np.float32(np.inf))))
                             assert st["reachable"] == reach, what
                             assert st["updates"] >= reach - 1, what
+
+
+# ------------------------------------------- run-error contract (§8(b)) ----
+def _overflow_graph():
+    """Symmetric graph whose shortest distance to vertex 38 overflows u32:
+    0 -(1)- leaves 1..16 (light at Delta = 2^31), leaf 1 -(0xC0000000)- 20
+    vertices 17..36 (heavy), 17 -(0xC0000000)- 37 -(1)- 38. Buckets 0 and 1
+    hold >= V/16 entries, so with PULL_SYMMETRIC the pull phases 2&3 see the
+    overflowing candidate; with push phases 2&3 the push relaxation does.
+    Vertices 39 -(2)- 40 form a separate component with no overflow."""
+    big = 0xC0000000
+    e = [(0, i, 1) for i in range(1, 17)] + [(1, 16 + j, big) for j in range(1, 21)]
+    e += [(17, 37, big), (37, 38, 1), (39, 40, 2)]
+    arcs = [(u, v, w) for u, v, w in e] + [(v, u, w) for u, v, w in e]
+    return csr_from_arcs(41, arcs)
+
+
+@pytest.mark.parametrize("pull", [0, 1])
+@pytest.mark.parametrize("path", ["sync", "async", "batch"])
+def test_overflow_reported_on_every_path(sssp, pull, path):
+    """u32 overflow (R12) is reported by sssp_distances, by sssp_wait after
+    sssp_distances_async, and by sssp_run_batch -- with push and with pull
+    phases 2&3 -- and a later clean run reports OK again."""
+    import torch
+
+    row, col, w = _overflow_graph()
+    delta = 2.0 ** 31
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, pull)
+        with pytest.raises(sssp.SSSPError) as e:
+            if path == "sync":
+                G.sssp(0, delta)
+            elif path == "async":
+                G.run(0, delta)
+                G.distances_async(torch.empty(41, dtype=torch.int32).pin_memory())
+                G.wait()
+            else:
+                out = torch.empty((2, 41), dtype=torch.int32, device="cuda")
+                G.run_batch([5, 0], delta, out)
+        assert e.value.status == sssp.SSSP_ERR_OVERFLOW, path
+        # the error was reported once and cleared: a clean run (the other component) is OK
+        d = G.sssp(39, 1)
+        assert d[40] == 2 and d[39] == 0 and d[0] == INF
+        G.run(39, 1)
+        G.distances_async(torch.empty(41, dtype=torch.int32).pin_memory())
+        G.wait()
+
+
+def test_overflow_of_unreported_run_surfaces_at_wait(sssp):
+    """Errors accumulate per handle: an overflowing run followed by a clean run
+    (neither reported) still makes the next sssp_wait fail."""
+    row, col, w = _overflow_graph()
+    with sssp.Graph(row, col, w) as G:
+        G.run(0, 2.0 ** 31)
+        G.run(39, 1)
+        with pytest.raises(sssp.SSSPError) as e:
+            G.wait()
+        assert e.value.status == sssp.SSSP_ERR_OVERFLOW
+        G.wait()  # cleared
+
+
+def test_multi_source_overflow_in_first_group(sssp):
+    """sssp_run_multi with 64 sources: the overflow happens only in group 0
+    (source 0); group 1's clean run must not wipe it."""
+    import torch
+
+    row, col, w = _overflow_graph()
+    g2 = gen.kronecker(8, 8, seed=3)  # second component, small weights
+    V1 = 41
+    row2 = np.concatenate([row, g2.row[1:] + row[-1]]).astype(np.int64)
+    col2 = np.concatenate([col, g2.col + V1]).astype(np.uint32)
+    w2 = np.concatenate([w, g2.w]).astype(np.uint32)
+    V = V1 + g2.V
+    other = [V1 + int(s) for s in gen.sample_sources(g2, 63, seed=1)]
+    srcs = [0] + other
+    with sssp.Graph(row2, col2, w2) as G:
+        out = torch.empty((64, V), dtype=torch.int32, device="cuda")
+        with pytest.raises(sssp.SSSPError) as e:
+            G.run_multi(srcs, 2.0 ** 31, out)
+        assert e.value.status == sssp.SSSP_ERR_OVERFLOW
+        G.run_multi(other, 16, out[:63])  # clean
+
+
+def test_pull_symmetric_is_checked(sssp):
+    """SSSP_PARAM_PULL_SYMMETRIC is verified, not trusted: a directed
+    Kronecker graph (one arc per edge, R13) is reported asymmetric and the
+    pull cannot be enabled; the generators' symmetrised graphs pass."""
+    gd = gen.kronecker(11, 16, seed=5, symmetrize=False)
+    gs = gen.kronecker(11, 16, seed=5)
+    s = int(gen.sample_sources(gd, 1, seed=1)[0])
+    exp = oracle.dijkstra(gd.row, gd.col, gd.w, s)
+    with sssp.Graph(gd.row, gd.col, gd.w) as G:
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)  # not reordered yet: checked at run
+        G.reorder()
+        assert not G.is_symmetric()
+        with pytest.raises(sssp.SSSPError) as e:
+            G.run(s, 16)
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 0)
+        assert_same(G.sssp(s, 16), exp, "directed graph, push phases 2&3")
+        with pytest.raises(sssp.SSSPError) as e:
+            G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        assert e.value.status == sssp.SSSP_ERR_INVALID_STATE
+    with sssp.Graph(gs.row, gs.col, gs.w) as G:
+        with pytest.raises(sssp.SSSPError):
+            G.is_symmetric()  # needs the weight-sorted layout
+        G.reorder()
+        assert G.is_symmetric()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+    # one reverse arc with a different weight breaks symmetry
+    row, col, w = csr_from_arcs(3, [(0, 1, 4), (1, 0, 5), (1, 2, 1), (2, 1, 1)])
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        assert not G.is_symmetric()
+    # multiplicities must match: (0,1,4) twice one way, once the other
+    row, col, w = csr_from_arcs(2, [(0, 1, 4), (0, 1, 4), (1, 0, 4)])
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        assert not G.is_symmetric()
+    row, col, w = csr_from_arcs(2, [(0, 1, 4), (0, 1, 4), (1, 0, 4), (1, 0, 4), (0, 0, 3)])
+    with sssp.Graph(row, col, w) as G:
+        G.reorder()
+        assert G.is_symmetric()

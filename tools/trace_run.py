@@ -11,7 +11,7 @@ import numpy as np  # noqa: E402
 
 import gen  # noqa: E402
 
-NAMES = {0: "P1", 1: "P2", 2: "RC", 3: "RF", 4: "SL", 5: "SH", 99: "start"}
+NAMES = {0: "P1", 1: "P2", 2: "RC", 3: "RF", 4: "SL", 5: "SH", 6: "P2C", 7: "MG", 9: "PL", 99: "start"}
 
 
 def main():
@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--no-reorder", action="store_true")
     ap.add_argument("--param", action="append", default=[])
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--samples", action="store_true", help="phase-1 claim samples of the last run per bucket")
     a = ap.parse_args()
     import torch
     import paper_conf_icppw_zhangczsdhay23_b200 as sssp
@@ -59,12 +60,44 @@ def main():
                 n = pr["lat_n"]
                 print(f"    task latency (cycles, warp 0): arc={pr['lat_arc']/n:.0f} probe={pr['lat_probe']/n:.0f} "
                       f"atom={pr['lat_atom']/n:.0f} stage={pr['lat_stage']/n:.0f} atomics_issued={pr['atoms']}", flush=True)
+        if a.samples:
+            smp = G.samples()
+            tr0 = G.trace()
+            t0 = tr0[0]["t_us"] if tr0 else 0.0
+            import collections
+            byb = collections.defaultdict(list)
+            for x in smp:
+                byb[x["cur"]].append(x)
+            base = min((x["t_ns"] for x in smp), default=0)
+            print(f"  samples: {len(smp)} (every 37th CTA's phase-1 claims); per bucket, 50 us windows: "
+                  "t_us  claims  items  tail(max)  pend(max)")
+            for b in sorted(byb):
+                xs = sorted(byb[b], key=lambda x: x["t_ns"])
+                tb = xs[0]["t_ns"]
+                win = collections.defaultdict(list)
+                for x in xs:
+                    win[int((x["t_ns"] - tb) / 50e3)].append(x)
+                print(f"   bucket {b}: {len(xs)} claims over {(xs[-1]['t_ns']-tb)/1e3:.1f} us "
+                      f"(from +{(tb-base)/1e3:.1f} us)")
+                if len(xs) > 20:
+                    for w in sorted(win):
+                        ys = win[w]
+                        print(f"      {w*50:6d}  {len(ys):5d}  {sum(y['claimed'] for y in ys):7d}  "
+                              f"{max(y['tail'] for y in ys):9d}  {max(y['pend'] for y in ys):9d}")
         if not a.quiet:
             tr = G.trace()
             prev = 0.0
+            prev_rel = 0.0
+            print("  columns: t(last arrival)  (+since previous)  kind ... | work = first arrival - previous "
+                  "release, drain = last - first arrival, step = release - last arrival")
             for e in tr:
+                if "t_first_us" in e and e["which"] != 8:
+                    print(f"      | work {e['t_first_us']-prev_rel:8.1f}  drain {e['t_us']-e['t_first_us']:7.1f}  "
+                          f"step {e['t_rel_us']-e['t_us']:5.1f} us")
+                    prev_rel = e["t_rel_us"]
                 print(f"  {e['t_us']:10.1f} us (+{e['t_us']-prev:8.1f})  {NAMES.get(e['which'], e['which']):5s} "
-                      f"cur={e['cur']} tail={e['tail']} mode={e['mode']}")
+                      f"cur={e['cur']} tail={e['tail']} mode={e['mode']}"
+                      + (f"  closed b{e['closed_b']} C={e['closed_c']}" if e.get("closed_b", 0xFFFFFFFF) != 0xFFFFFFFF else ""))
                 prev = e["t_us"]
 
 
