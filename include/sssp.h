@@ -218,7 +218,7 @@ typedef enum {
                                       frontier level, the paper's BL); 0 the
                                       bucket-aware asynchronous phase 1 (BASYN) [0] */
     SSSP_PARAM_P2_EDGE_BALANCED = 7, /* phases 2&3 with equal heavy arcs per warp
-                                      for buckets with >= value settled entries; smaller
+                                      for buckets with >= value (< 2^23) settled entries; smaller
                                       buckets (and -1 = never) relax heavy arcs through the
                                       phase-1 vertex bins [-1] */
     SSSP_PARAM_ADAPTIVE_DELTA = 8, /* NEXT-1, Eq. (1)-(2) P:1006-1028 (Alg. 2 l.11): 0 fixed
@@ -301,11 +301,15 @@ typedef struct sssp_trace_entry {
 sssp_status sssp_get_trace(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
                            int64_t* n_entries);
 
-/* Diagnostics of the last run: phase-1 claim samples of every 37th CTA, in
- * time order per CTA (which = 100; t_ns = %globaltimer; cur = bucket; tail =
- * queue entries pushed so far; far_min = pending entries; mode = entries
+/* Diagnostics of the last run: samples of every 37th CTA, in time order per
+ * CTA. which = 100, a phase-1 claim: t_ns = %globaltimer; cur = bucket; tail
+ * = queue entries pushed so far; far_min = pending entries; mode = entries
  * claimed (0: the phase ended); pad = first claimed position; closed_b = CTA;
- * closed_c = 1 for a CTA-local batch). Up to 16384 entries. */
+ * closed_c = 1 for a CTA-local batch. which = 101, a processed batch: tail =
+ * warp tasks, mode = thread-bin tasks, far_min = range-list entries, t_first
+ * / t_rel / pad = SM cycles staging / in warp 0's task loop / waiting for the
+ * other warps and flushing, closed_c = 10 * phase + source (batch records only
+ * in builds with -DSSSP_BATCH_SAMPLES=1). Up to 16384. */
 sssp_status sssp_get_samples(sssp_graph_t g, sssp_trace_entry* out, int64_t max_entries,
                              int64_t* n_entries);
 

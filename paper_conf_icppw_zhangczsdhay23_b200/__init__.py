@@ -289,9 +289,17 @@ def sssp_get_samples(h, max_entries=16384):
     _check(_lib.sssp_get_samples(h, buf, max_entries, ctypes.byref(n)), "sssp_get_samples")
     m = min(n.value, max_entries)
     t0 = min((buf[i].t_ns for i in range(m)), default=0)
-    return [dict(t_us=(buf[i].t_ns - t0) / 1e3, t_ns=buf[i].t_ns, cur=buf[i].cur, tail=buf[i].tail,
-                 claimed=buf[i].mode, pend=buf[i].far_min, pos=buf[i].pad, cta=buf[i].closed_b)
-            for i in range(m)]
+    out = []
+    for i in range(m):
+        b = buf[i]
+        if b.which == 101:  # batch record: SM cycles of stage / warp-0 task loop / tail
+            out.append(dict(kind="batch", t_us=(b.t_ns - t0) / 1e3, t_ns=b.t_ns, cur=b.cur, tasks=b.tail,
+                            tb_tasks=b.mode, ranges=b.far_min, cyc_stage=b.t_first, cyc_task=b.t_rel,
+                            cyc_tail=b.pad, cta=b.closed_b, src=b.closed_c))
+        else:
+            out.append(dict(kind="claim", t_us=(b.t_ns - t0) / 1e3, t_ns=b.t_ns, cur=b.cur, tail=b.tail,
+                            claimed=b.mode, pend=b.far_min, pos=b.pad, cta=b.closed_b))
+    return out
 
 
 def sssp_get_profile(h):

@@ -58,6 +58,9 @@ constexpr u32 HUB_CHUNK = 4096;
 #ifndef SSSP_LAT
 #define SSSP_LAT 0  // per-stage latency accounting in the task loop (diagnostics build)
 #endif
+#ifndef SSSP_BATCH_SAMPLES
+#define SSSP_BATCH_SAMPLES 0  // per-batch stage/task/tail cycles in sssp_get_samples (diagnostics build)
+#endif
 constexpr int UNROLL = SSSP_UNROLL;
 #ifndef SSSP_IPT
 #define SSSP_IPT 2  // queue items decoded per thread per phase-1 batch
@@ -216,7 +219,7 @@ struct Params {
   u32 claim_max;
   // ablation flags (bit 0 ADWL: adaptive thread/warp/CTA bins + hub chunks, 0 = thread per
   // vertex; bit 1 SYNC: level-synchronous phase 1, a grid barrier per frontier level = BL;
-  // bit 2 EB: edge-balanced phase 2 for settled ranges of >= flags >> 8 entries;
+  // bit 2 EB: edge-balanced phase 2 for settled ranges of >= (flags >> 8) & 0x7FFFFF entries;
   // bit 7 PULL: pull-style phases 2&3 for large buckets (symmetric graphs, PRO; f32 graphs
   // then carry Delta's bits in delta_u);
   // bits 3/4 adaptive Delta reading A/B (NEXT-1); bit 5 f32 weights (theta level bits)).
@@ -241,6 +244,17 @@ constexpr u32 LOCAL_LIM_MASK = 4095u;
 static_assert(BATCH < LOCAL_CHASE, "claim_max must fit below the LOCAL_CHASE bit");
 static_assert(LOC_CAP <= LOCAL_LIM_MASK, "local-chase limit field too narrow for LOC_CAP");
 
+// What pb_flush needs, kept in shared memory (Smem::fctx) so the out-of-line call takes no
+// parameter registers.
+struct FlushCtx {
+  SlotCtl* sc;
+  u64* items;
+  Ctl* ctl;
+  u32* xd;
+  u32 cap, kmask, delta_u;
+  float inv_delta;
+};
+
 struct Smem {
   // Task pool of one batch. Tasks [0, S): 128-arc slices of each warp's
   // thread bin (small vertices, arcs spread by a warp prefix sum); tasks
@@ -262,6 +276,8 @@ struct Smem {
   u32 rl_n, rl_tasks, task_next;
   u64 pb[DS_WARPS][PB_CAP];  // staged pushes (d << 32 | v), bucket resolved at flush
   u32 pb_n[DS_WARPS];
+  u32 fc[DS_WARPS][64];      // pb_flush: entries per ring slot, then each slot's next position
+  FlushCtx fctx;
   unsigned long long st[ST_N];
   u32 claim_h, claim_n, claim_src;
   // CTA-local chase (LOCAL_CHASE): phase-1 pushes into the current bucket kept in shared
@@ -360,15 +376,6 @@ __device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
 // distinct bucket queue (tail and pend in one atomicAdd). Entries beyond the
 // ring horizon or a full queue are dropped and recorded in far_min. In the
 // sweep fall-back (nearb != NONE) entries of bucket nearb mark xd[] instead.
-// What pb_flush needs, passed by value (48 B) to the out-of-line call.
-struct FlushCtx {
-  SlotCtl* sc;
-  u64* items;
-  Ctl* ctl;
-  u32* xd;
-  u32 cap, kmask, delta_u;
-  float inv_delta;
-};
 
 template <bool F32>
 __device__ __forceinline__ u32 bucket_of_f(const FlushCtx& p, u32 d) {
@@ -380,19 +387,28 @@ __device__ __forceinline__ u32 bucket_of_f(const FlushCtx& p, u32 d) {
   }
 }
 
+// Publish warp w's staged pushes. Entries beyond the ring horizon or a full queue are
+// dropped and recorded in far_min; in the sweep fall-back (nearb != NONE) entries of bucket
+// nearb mark xd[] instead; with the CTA-local chase, current-bucket entries stay in the CTA.
+// Reservations (tail and pend in one atomicAdd on the slot's control word): every CTA
+// pushing into a bucket hits that one word, and on C4 the peak bucket's word saturated the
+// L2's same-address atomic rate (ncu: ~28 % of all stall samples waited on it). So a flush
+// of more than 32 entries makes two passes -- classify and count per ring slot, one
+// atomicAdd per non-empty slot (all in flight together), then place -- instead of one
+// reservation per slot per 32 entries; a flush of <= 32 entries (thin frontiers, C2) keeps
+// the single pass and its shorter latency.
 template <bool F32>
-__device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, u32 nearb) {
+__device__ __noinline__ void pb_flush_impl(Smem& sm, u32 lim, u32 nearb) {
+  const FlushCtx& p = sm.fctx;
   const u32 lane = lane_id(), w = threadIdx.x >> 5;
   const u32 n = sm.pb_n[w];
   if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)n);
-  for (u32 i0 = 0; i0 < n; i0 += 32) {
-    const u32 i = i0 + lane;
-    bool ok = i < n;
-    const u64 e = ok ? sm.pb[w][i] : 0ULL;
+  const u32 c0 = sm.cur, ce = sm.cur_end;
+  // entry -> (keep for the global queue?, ring slot, bucket); handles the dropped cases
+  auto classify = [&](u64 e, bool ok, u32& x, u32& slot) -> bool {
     const u32 v = (u32)e, nd = (u32)(e >> 32);
-    const u32 x = ok ? bucket_of_f<F32>(p, nd) : 0u;
-    const u32 c0 = sm.cur;
-    const bool in_cur = x - c0 < sm.cur_end - c0;  // current bucket [cur, cur_end): its queue is slot cur
+    x = ok ? bucket_of_f<F32>(p, nd) : 0u;
+    const bool in_cur = x - c0 < ce - c0;  // current bucket [cur, cur_end): its queue is slot cur
     if (ok && nearb != NONE && in_cur) {
       st_relaxed_u32(p.xd + v, NONE);
       st_relaxed_u32(&p.ctl->changed, 1u);
@@ -417,22 +433,77 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
       atomicMin(&p.ctl->far_min, x);
       ok = false;
     }
+    slot = (in_cur ? c0 : x) & p.kmask;
+    return ok;
+  };
+  auto place = [&](u64 e, u32 x, u32 slot, u32 idx) {
+    if (idx < p.cap) {
+      st_relaxed_u64(p.items + (u64)slot * p.cap + idx, e);
+    } else {  // queue full: undo the pending count, recover later
+      atomicAdd(&p.sc[slot].word, ~0ULL);
+      atomicMin(&p.ctl->far_min, x);
+    }
+  };
+  if (n <= 32) {
+    const bool has = lane < n;
+    const u64 e = has ? sm.pb[w][lane] : 0ULL;
+    u32 x, slot;
+    const bool ok = classify(e, has, x, slot);
     const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
     if (ok) {
-      const u32 s = (in_cur ? c0 : x) & p.kmask;
-      const u32 peers = __match_any_sync(m, s);
+      const u32 peers = __match_any_sync(m, slot);
       const u32 leader = __ffs(peers) - 1;
       const u32 cnt = __popc(peers);
       u64 old = 0;
-      if (lane == leader) old = atomicAdd(&p.sc[s].word, ((u64)cnt << 32) | cnt);
+      if (lane == leader) old = atomicAdd(&p.sc[slot].word, ((u64)cnt << 32) | cnt);
       old = __shfl_sync(peers, old, leader);
-      const u32 idx = (u32)(old >> 32) + __popc(peers & lanemask_lt());
-      if (idx < p.cap) {
-        st_relaxed_u64(p.items + (u64)s * p.cap + idx, e);
-      } else {  // queue full: undo the pending count, recover later
-        atomicAdd(&p.sc[s].word, ~0ULL);
-        atomicMin(&p.ctl->far_min, x);
+      place(e, x, slot, (u32)(old >> 32) + __popc(peers & lanemask_lt()));
+    }
+  } else {
+    u32* fc = sm.fc[w];
+    const u32 K = p.kmask + 1;
+    for (u32 k = lane; k < K; k += 32) fc[k] = 0;
+    __syncwarp();
+    for (u32 i0 = 0; i0 < n; i0 += 32) {  // pass 1: classify, count per slot
+      const u32 i = i0 + lane;
+      const bool has = i < n;
+      const u64 e = has ? sm.pb[w][i] : 0ULL;
+      u32 x, slot;
+      const bool ok = classify(e, has, x, slot);
+      if (has && !ok) sm.pb[w][i] = SENTINEL;  // handled (or dropped) here
+      const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
+      if (ok) {
+        const u32 peers = __match_any_sync(m, slot);
+        if (lane == __ffs(peers) - 1) fc[slot] += __popc(peers);
       }
+      __syncwarp();
+    }
+    for (u32 k = lane; k < K; k += 32) {  // one reservation per non-empty slot
+      const u32 c = fc[k];
+      if (c) fc[k] = (u32)(atomicAdd(&p.sc[k].word, ((u64)c << 32) | c) >> 32);
+    }
+    __syncwarp();
+    for (u32 i0 = 0; i0 < n; i0 += 32) {  // pass 2: place at the reserved positions
+      const u32 i = i0 + lane;
+      const u64 e = i < n ? sm.pb[w][i] : SENTINEL;
+      const bool ok = e != SENTINEL;
+      u32 x = 0, slot = 0;
+      if (ok) {
+        x = bucket_of_f<F32>(p, (u32)(e >> 32));
+        slot = (x - c0 < ce - c0 ? c0 : x) & p.kmask;
+      }
+      const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
+      u32 base = 0, peers = 0;
+      if (ok) {
+        peers = __match_any_sync(m, slot);
+        base = fc[slot];
+      }
+      __syncwarp();
+      if (ok) {
+        if (lane == __ffs(peers) - 1) fc[slot] = base + __popc(peers);
+        place(e, x, slot, base + __popc(peers & lanemask_lt()));
+      }
+      __syncwarp();
     }
   }
   __syncwarp();
@@ -442,8 +513,7 @@ __device__ __noinline__ void pb_flush_impl(const FlushCtx p, Smem& sm, u32 lim, 
 
 template <bool F32>
 __device__ __forceinline__ void pb_flush(const Params& p, Smem& sm, u32 lim, u32 nearb) {
-  const FlushCtx f = {p.sc, p.items, p.ctl, p.xd, p.cap, p.kmask, p.delta_u, p.inv_delta};
-  pb_flush_impl<F32>(f, sm, lim, nearb);
+  pb_flush_impl<F32>(sm, lim, nearb);
 }
 
 // Stage up to UNROLL pushes per lane into the warp's buffer (all 32 lanes).
@@ -874,7 +944,28 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   }
   if (sm.pb_n[w]) pb_flush<F32>(p, sm, lim, nearb);  // publish before reporting completion
   __syncthreads();
-  if (tid == 0) sm.st[ST_P_TAIL] += (unsigned long long)(clock64() - t_task);
+  if (tid == 0) {
+    const long long t_end = clock64();
+    sm.st[ST_P_TAIL] += (unsigned long long)(t_end - t_task);
+    if (SSSP_BATCH_SAMPLES && blockIdx.x % SAMPLE_EVERY == 0) {  // batch timeline (which = 101)
+      const u32 k = atomicAdd(&p.ctl->sample_n, 1u);
+      if (k < SAMPLE_CAP) {
+        TraceEnt e;
+        e.t_ns = globaltimer();
+        e.which = 101;
+        e.cur = sm.cur;
+        e.tail = ntask;
+        e.mode = S;
+        e.far_min = nl;
+        e.pad = (u32)(t_end - t_task);
+        e.closed_b = blockIdx.x;
+        e.closed_c = PH * 10 + src;
+        e.t_first = (u64)(t_pool - t_enter);
+        e.t_rel = (u64)(t_task - t_pool);
+        p.trace[TRACE_CAP + k] = e;
+      }
+    }
+  }
 }
 
 // --------------------------------------------------------- grid barrier ---
@@ -984,7 +1075,7 @@ __device__ void decide(const Params& p, u32 which) {
       c->mode = MODE_PULL;
       return;
     }
-    if ((p.flags & 4u) && tail - b >= (p.flags >> 8)) {  // edge-balanced phase 2
+    if ((p.flags & 4u) && tail - b >= ((p.flags >> 8) & 0x7FFFFFu)) {  // edge-balanced phase 2
       c->hub_word = 0;
       c->p2_head = 0;
       c->mode = MODE_P2_COMPACT;
@@ -1126,6 +1217,12 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
       const u64 t = globaltimer();
       decide(p, which);
       volatile Ctl* vc = c;
+      const u64 t_first = vc->t_first;
+      vc->t_first = ~0ULL;
+      const u64 t_rel = globaltimer();
+      grid_release(&c->bar_gen, target);
+      // The record is written after the release, off the critical path: what it reads was
+      // set by decide() and stays put until the next barrier, which this thread must reach.
       const u32 tn = vc->trace_n;
       if (tn < TRACE_CAP) {
         TraceEnt e;
@@ -1138,13 +1235,11 @@ __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
         e.pad = vc->cur_end;
         e.closed_b = vc->closed_b;
         e.closed_c = vc->closed_c;
-        e.t_first = vc->t_first;
-        e.t_rel = globaltimer();
+        e.t_first = t_first;
+        e.t_rel = t_rel;
         p.trace[tn] = e;
         vc->trace_n = tn + 1;
       }
-      vc->t_first = ~0ULL;
-      grid_release(&c->bar_gen, target);
     } else {
       grid_wait(&c->bar_gen, target);
     }
@@ -1971,6 +2066,7 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
   if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
   if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
+    sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.cap, p.kmask, p.delta_u, p.inv_delta};
     sm.loc_n = 0;
     sm.loc_on = 0;
     volatile Ctl* vc = p.ctl;

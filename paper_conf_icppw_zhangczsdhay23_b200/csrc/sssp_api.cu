@@ -319,7 +319,7 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       g->p_sync = v;
       return SSSP_OK;
     case SSSP_PARAM_P2_EDGE_BALANCED:
-      if (v < -1 || v > 0xFFFFFF) return fail(SSSP_ERR_INVALID_ARGUMENT, "p2 edge-balanced threshold in [-1, 2^24)");
+      if (v < -1 || v > 0x7FFFFF) return fail(SSSP_ERR_INVALID_ARGUMENT, "p2 edge-balanced threshold in [-1, 2^23)");
       g->p_p2eb = v;
       return SSSP_OK;
     case SSSP_PARAM_ADAPTIVE_DELTA:
@@ -761,7 +761,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   p.p2o = g->p2o;
   p.flags = (g->p_adwl ? 1u : 0u) | (g->p_sync ? 2u : 0u);
   // edge-balanced phase 2 (not in the static thread-per-vertex ablation)
-  if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0xFFFFFF) << 8);
+  if (g->p_p2eb >= 0 && g->p_adwl) p.flags |= 4u | ((u32)std::min<i64>(g->p_p2eb, 0x7FFFFF) << 8);
   if (adapt) p.flags |= (dp.ai.mode == 2 ? 16u : 8u) | (pro ? 64u : 0u);
   if (f32) p.flags |= 32u;
   if (g->p_pull && pro && !adapt && (f32 ? dp.inv != 0.f : dp.delta_u != 0xFFFFFFFFu)) {  // symmetric, checked

@@ -66,8 +66,16 @@ def main():
             t0 = tr0[0]["t_us"] if tr0 else 0.0
             import collections
             byb = collections.defaultdict(list)
+            bat = collections.defaultdict(list)
             for x in smp:
-                byb[x["cur"]].append(x)
+                (byb if x.get("kind", "claim") == "claim" else bat)[x["cur"]].append(x)
+            print("  batches per bucket (sampled CTAs): n  tasks/batch  stage/task/tail kcycles per batch")
+            for b in sorted(bat):
+                xs = bat[b]
+                n = len(xs)
+                print(f"   bucket {b}: {n:5d}  {sum(x['tasks'] for x in xs)/n:7.1f}  "
+                      f"{sum(x['cyc_stage'] for x in xs)/n/1e3:6.2f} {sum(x['cyc_task'] for x in xs)/n/1e3:6.2f} "
+                      f"{sum(x['cyc_tail'] for x in xs)/n/1e3:6.2f}")
             base = min((x["t_ns"] for x in smp), default=0)
             print(f"  samples: {len(smp)} (every 37th CTA's phase-1 claims); per bucket, 50 us windows: "
                   "t_us  claims  items  tail(max)  pend(max)")
