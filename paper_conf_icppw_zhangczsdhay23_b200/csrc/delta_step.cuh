@@ -47,7 +47,7 @@ constexpr u32 BIN_WARP = 32;     // beta
 constexpr u32 BIN_CTA = 256;     // alpha
 constexpr u32 HUB_CHUNK = 4096;
 #ifndef SSSP_UNROLL
-#define SSSP_UNROLL 4
+#define SSSP_UNROLL 2  // arcs per lane per warp task (B200 A/B: 2 beats 4 and 1 on C4 and C3, profiles/r02)
 #endif
 #ifndef SSSP_PROBE_L1
 #define SSSP_PROBE_L1 1  // dist probes through L1 (a stale value is a safe filter)
@@ -57,6 +57,9 @@ constexpr u32 HUB_CHUNK = 4096;
 #endif
 #ifndef SSSP_LAT
 #define SSSP_LAT 0  // per-stage latency accounting in the task loop (diagnostics build)
+#endif
+#ifndef SSSP_DEFER_ATOMICS
+#define SSSP_DEFER_ATOMICS 1  // relaxations' atomicMin issued by pb_flush, a staged batch at once
 #endif
 #ifndef SSSP_BATCH_SAMPLES
 #define SSSP_BATCH_SAMPLES 0  // per-batch stage/task/tail cycles in sssp_get_samples (diagnostics build)
@@ -83,6 +86,7 @@ constexpr int IPT_MAX = IPT > IPT2 ? IPT : IPT2;
 constexpr u64 SENTINEL = ~0ULL;
 constexpr u32 NONE = 0xFFFFFFFFu;
 constexpr u32 CHUNK_FLAG = 0x80000000u;
+constexpr u32 APPLIED_FLAG = 0x80000000u;  // in a staged push's vertex field (V < 2^31), see stage_pushes
 
 enum : u32 {
   MODE_PHASE1 = 0,
@@ -234,7 +238,7 @@ constexpr u32 BATCH = DS_THREADS * IPT;        // queue items per phase-1 CTA ba
 constexpr u32 BATCH_MAX = DS_THREADS * IPT_MAX;
 constexpr u32 SB_CAP = 32 * IPT_MAX;           // thread-bin entries per warp
 #ifndef SSSP_PB_CAP
-#define SSSP_PB_CAP 256u
+#define SSSP_PB_CAP 128u  // (128 beats 256 and 64, profiles/r02)
 #endif
 constexpr u32 PB_CAP = SSSP_PB_CAP;  // staged pushes per warp (>= 32 * UNROLL)
 constexpr u32 LOC_CAP = BATCH;       // CTA-local chase list: one phase-1 batch
@@ -251,6 +255,7 @@ struct FlushCtx {
   u64* items;
   Ctl* ctl;
   u32* xd;
+  u32* dist;
   u32 cap, kmask, delta_u;
   float inv_delta;
 };
@@ -396,13 +401,47 @@ __device__ __forceinline__ u32 bucket_of_f(const FlushCtx& p, u32 d) {
 // of more than 32 entries makes two passes -- classify and count per ring slot, one
 // atomicAdd per non-empty slot (all in flight together), then place -- instead of one
 // reservation per slot per 32 entries; a flush of <= 32 entries (thin frontiers, C2) keeps
-// the single pass and its shorter latency.
+// the single pass and its shorter latency. (Measured on C4: one flush waiting a single round
+// trip -- reservations issued while the candidates' atomics are in flight, dead entries for
+// the losers -- was 7 % slower than this: profiles/r02/ab_flush_merged_negative.txt.)
 template <bool F32>
 __device__ __noinline__ void pb_flush_impl(Smem& sm, u32 lim, u32 nearb) {
   const FlushCtx& p = sm.fctx;
   const u32 lane = lane_id(), w = threadIdx.x >> 5;
   const u32 n = sm.pb_n[w];
-  if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)n);
+  {  // pass 0: the staged relaxations' atomicMin (Alg. 1 l.3, SSSP_DEFER_ATOMICS), four rounds
+     // in flight; an entry that did not lower dist[v] is dropped (SENTINEL), an applied one
+     // (stage_pushes<.., true>) only loses its flag
+    const u64 pol_keep = policy_evict_last();
+    constexpr int AR = 4;
+    u32 nsurv = 0;
+    for (u32 i0 = 0; i0 < n; i0 += 32 * AR) {
+      u64 e[AR];
+      u32 old[AR];
+#pragma unroll
+      for (int r = 0; r < AR; ++r) {
+        const u32 i = i0 + r * 32 + lane;
+        e[r] = i < n ? sm.pb[w][i] : SENTINEL;
+        const bool need = e[r] != SENTINEL && !((u32)e[r] & APPLIED_FLAG);
+        old[r] = atomic_min_keep(p.dist + (u32)e[r], (u32)(e[r] >> 32), need, pol_keep);
+      }
+#pragma unroll
+      for (int r = 0; r < AR; ++r) {
+        if (e[r] == SENTINEL) continue;
+        const u32 i = i0 + r * 32 + lane;
+        const bool applied = ((u32)e[r] & APPLIED_FLAG) != 0;
+        if (applied || (u32)(e[r] >> 32) < old[r]) {
+          if (applied) sm.pb[w][i] = e[r] & ~(u64)APPLIED_FLAG;
+          ++nsurv;
+        } else {
+          sm.pb[w][i] = SENTINEL;
+        }
+      }
+    }
+    nsurv = __reduce_add_sync(SSSP_FULL_MASK, nsurv);
+    if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)nsurv);
+    __syncwarp();
+  }
   const u32 c0 = sm.cur, ce = sm.cur_end;
   // entry -> (keep for the global queue?, ring slot, bucket); handles the dropped cases
   auto classify = [&](u64 e, bool ok, u32& x, u32& slot) -> bool {
@@ -445,8 +484,9 @@ __device__ __noinline__ void pb_flush_impl(Smem& sm, u32 lim, u32 nearb) {
     }
   };
   if (n <= 32) {
-    const bool has = lane < n;
-    const u64 e = has ? sm.pb[w][lane] : 0ULL;
+    const u64 e0 = lane < n ? sm.pb[w][lane] : SENTINEL;
+    const bool has = e0 != SENTINEL;
+    const u64 e = has ? e0 : 0ULL;
     u32 x, slot;
     const bool ok = classify(e, has, x, slot);
     const u32 m = __ballot_sync(SSSP_FULL_MASK, ok);
@@ -466,8 +506,9 @@ __device__ __noinline__ void pb_flush_impl(Smem& sm, u32 lim, u32 nearb) {
     __syncwarp();
     for (u32 i0 = 0; i0 < n; i0 += 32) {  // pass 1: classify, count per slot
       const u32 i = i0 + lane;
-      const bool has = i < n;
-      const u64 e = has ? sm.pb[w][i] : 0ULL;
+      const u64 e0 = i < n ? sm.pb[w][i] : SENTINEL;
+      const bool has = e0 != SENTINEL;
+      const u64 e = has ? e0 : 0ULL;
       u32 x, slot;
       const bool ok = classify(e, has, x, slot);
       if (has && !ok) sm.pb[w][i] = SENTINEL;  // handled (or dropped) here
@@ -516,8 +557,10 @@ __device__ __forceinline__ void pb_flush(const Params& p, Smem& sm, u32 lim, u32
   pb_flush_impl<F32>(sm, lim, nearb);
 }
 
-// Stage up to UNROLL pushes per lane into the warp's buffer (all 32 lanes).
-template <bool F32>
+// Stage up to UNROLL pushes per lane into the warp's buffer (all 32 lanes). APPLIED: dist[v]
+// already holds nd (the entry only needs queueing); otherwise the entry is a relaxation
+// candidate whose atomicMin pb_flush issues (SSSP_DEFER_ATOMICS).
+template <bool F32, bool APPLIED = true>
 __device__ __forceinline__ void stage_pushes(const Params& p, Smem& sm, u32 lim, u32 nearb,
                                              const bool (&want)[UNROLL], const u32 (&v)[UNROLL],
                                              const u32 (&nd)[UNROLL]) {
@@ -533,7 +576,7 @@ __device__ __forceinline__ void stage_pushes(const Params& p, Smem& sm, u32 lim,
   u32 base = sm.pb_n[w];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
-    if (want[k]) sm.pb[w][base + __popc(m[k] & lt)] = ((u64)nd[k] << 32) | v[k];
+    if (want[k]) sm.pb[w][base + __popc(m[k] & lt)] = ((u64)nd[k] << 32) | (v[k] | (APPLIED ? APPLIED_FLAG : 0u));
     base += __popc(m[k]);
   }
   __syncwarp();
@@ -596,6 +639,22 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
   }
   u32 n_atoms = 0;
 #endif
+  u32 vv[UNROLL];
+#if SSSP_DEFER_ATOMICS
+  // Alg. 1 l.2 here; the atomicMin of l.3 is issued by pb_flush for every staged candidate
+  // of the warp at once (a warp no longer waits one L2 atomic round trip per task)
+#pragma unroll
+  for (int k = 0; k < UNROLL; ++k) {
+    want[k] = want[k] && nd[k] < cur[k];
+    vv[k] = a[k].x;
+#if SSSP_LAT
+    n_atoms += want[k];
+#endif
+  }
+#if SSSP_LAT
+  st_add(sm, ST_ATOMS, n_atoms);
+#endif
+#else
   u32 old[UNROLL];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
@@ -608,19 +667,21 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
 #if SSSP_LAT
   st_add(sm, ST_ATOMS, n_atoms);
 #endif
-  u32 vv[UNROLL];
 #pragma unroll
   for (int k = 0; k < UNROLL; ++k) {
     want[k] = want[k] && nd[k] < old[k];
     vv[k] = a[k].x;
   }
+#endif
 #if SSSP_LAT
   if (threadIdx.x == 0) {
+#if !SSSP_DEFER_ATOMICS
     asm volatile("" ::"r"(old[0]), "r"(old[UNROLL - 1]));
+#endif
     t3 = clock64();
   }
 #endif
-  stage_pushes<F32>(p, sm, lim, nearb, want, vv, nd);
+  stage_pushes<F32, !SSSP_DEFER_ATOMICS>(p, sm, lim, nearb, want, vv, nd);
 #if SSSP_LAT
   if (threadIdx.x == 0) {
     const long long t4 = clock64();
@@ -666,6 +727,10 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   const bool sweep = src == SRC_SWEEP;
   const u32 nearb = sweep ? sm.cur : NONE;
   const long long t_enter = tid == 0 ? clock64() : 0;
+#if SSSP_LAT && SSSP_BATCH_SAMPLES
+  const unsigned long long lat0_probe = tid == 0 ? sm.st[ST_L_PROBE] : 0ULL;
+  const unsigned long long lat0_stage = tid == 0 ? sm.st[ST_L_STAGE] : 0ULL;
+#endif
   // ---- decode: all dist probes and row loads of the thread's items in flight at once
   u32 cls[N], beg[N], len[N], d[N];
   u32 cd[N];
@@ -955,8 +1020,13 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
         e.which = 101;
         e.cur = sm.cur;
         e.tail = ntask;
+#if SSSP_LAT
+        e.mode = (u32)(sm.st[ST_L_PROBE] - lat0_probe);  // warp 0's probe-wait cycles in this batch
+        e.far_min = (u32)(sm.st[ST_L_STAGE] - lat0_stage);  // ... and push-staging cycles
+#else
         e.mode = S;
         e.far_min = nl;
+#endif
         e.pad = (u32)(t_end - t_task);
         e.closed_b = blockIdx.x;
         e.closed_c = PH * 10 + src;
@@ -1747,7 +1817,8 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
   u32* out_n = &p.ctl->pull_n[osel];
   uint4* longq = reinterpret_cast<uint4*>(p.xd + ((3 * (u64)p.V + 3) & ~3ULL));  // 16-B aligned
   const u32 long_cap = p.V / 2;
-  constexpr int NV = UNROLL;  // candidates per lane in flight (stage_pushes takes UNROLL)
+  constexpr int NV = 4;       // candidates per lane in flight
+  static_assert(NV % UNROLL == 0, "pushes are staged UNROLL at a time");
   constexpr int PU = 2;       // heavy arcs per candidate per step
   u32 c_pull = 0, c_arcs = 0, c_in = 0;
   bool of = false;
@@ -1860,18 +1931,22 @@ __device__ void pull_phase(const Params& p, Smem& sm) {
         any |= act[k];
       }
     }
-    bool want[UNROLL];
-    u32 nd[UNROLL];
 #pragma unroll
-    for (int k = 0; k < NV; ++k) {
-      want[k] = v[k] != NONE && best[k] < dv[k];
-      nd[k] = best[k];
-      if (want[k]) {
-        atomicMin(p.dist + v[k], best[k]);  // v is this thread's alone during the pull
-        ++c_pull;
+    for (int k0 = 0; k0 < NV; k0 += UNROLL) {
+      bool want[UNROLL];
+      u32 vv[UNROLL], nd[UNROLL];
+#pragma unroll
+      for (int k = 0; k < UNROLL; ++k) {
+        want[k] = v[k0 + k] != NONE && best[k0 + k] < dv[k0 + k];
+        vv[k] = v[k0 + k];
+        nd[k] = best[k0 + k];
+        if (want[k]) {
+          atomicMin(p.dist + vv[k], nd[k]);  // v is this thread's alone during the pull
+          ++c_pull;
+        }
       }
+      stage_pushes<F32>(p, sm, lim, NONE, want, vv, nd);
     }
-    stage_pushes<F32>(p, sm, lim, NONE, want, v, nd);
   }
   if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
   if (!F32 && of) atomicOr(&p.ctl->err, ERR_OVERFLOW);
@@ -2066,7 +2141,7 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
   if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
   if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
-    sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.cap, p.kmask, p.delta_u, p.inv_delta};
+    sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.dist, p.cap, p.kmask, p.delta_u, p.inv_delta};
     sm.loc_n = 0;
     sm.loc_on = 0;
     volatile Ctl* vc = p.ctl;

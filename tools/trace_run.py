@@ -69,13 +69,15 @@ def main():
             bat = collections.defaultdict(list)
             for x in smp:
                 (byb if x.get("kind", "claim") == "claim" else bat)[x["cur"]].append(x)
-            print("  batches per bucket (sampled CTAs): n  tasks/batch  stage/task/tail kcycles per batch")
+            print("  batches per bucket (sampled CTAs): n  tasks/batch  stage/task/tail kcycles per batch"
+                  "  [LAT builds: warp-0 probe / staging kcycles per batch]")
             for b in sorted(bat):
                 xs = bat[b]
                 n = len(xs)
                 print(f"   bucket {b}: {n:5d}  {sum(x['tasks'] for x in xs)/n:7.1f}  "
                       f"{sum(x['cyc_stage'] for x in xs)/n/1e3:6.2f} {sum(x['cyc_task'] for x in xs)/n/1e3:6.2f} "
-                      f"{sum(x['cyc_tail'] for x in xs)/n/1e3:6.2f}")
+                      f"{sum(x['cyc_tail'] for x in xs)/n/1e3:6.2f}   "
+                      f"[{sum(x['tb_tasks'] for x in xs)/n/1e3:6.2f} {sum(x['ranges'] for x in xs)/n/1e3:6.2f}]")
             base = min((x["t_ns"] for x in smp), default=0)
             print(f"  samples: {len(smp)} (every 37th CTA's phase-1 claims); per bucket, 50 us windows: "
                   "t_us  claims  items  tail(max)  pend(max)")
