@@ -259,12 +259,8 @@ typedef enum {
                                       networks: thin frontiers; on dense ones the CTA-local
                                       depth-first order re-relaxes more). Same distances;
                                       0 = always through the global queue [1] */
-    SSSP_PARAM_LOCAL_LIMIT = 13,   /* local-chase entries a CTA keeps (1..512); pushes beyond
+    SSSP_PARAM_LOCAL_LIMIT = 13    /* local-chase entries a CTA keeps (1..512); pushes beyond
                                       go to the global queue, where idle CTAs can take them [512] */
-    SSSP_PARAM_BUCKET_DIV = 14     /* u32, fixed Delta: buckets of width Delta / value (1..16)
-                                      while light stays w < Delta (heavy arcs, w >= Delta, still
-                                      land in later buckets, so the result is exact). Same
-                                      distances; a schedule knob [1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

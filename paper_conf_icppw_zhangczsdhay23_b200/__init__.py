@@ -51,7 +51,6 @@ SSSP_PARAM_MULTI_HUB_DELAY = 10
 SSSP_PARAM_PULL_SYMMETRIC = 11
 SSSP_PARAM_LOCAL_CHASE = 12
 SSSP_PARAM_LOCAL_LIMIT = 13
-SSSP_PARAM_BUCKET_DIV = 14
 
 INF_U32 = 0xFFFFFFFF
 

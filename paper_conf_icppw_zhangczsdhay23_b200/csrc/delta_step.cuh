@@ -1100,6 +1100,83 @@ __device__ void adapt_next(const Params& p, u32 t_i, u32 c_i) {
   }
 }
 
+__device__ __forceinline__ uint4 ld_volatile_v4(const void* q) {
+  uint4 r;
+  asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(q)
+               : "memory");
+  return r;
+}
+
+// Closing a bucket after its phases 2&3 (SYNC_P2), fixed Delta: the same steps as the
+// general path in decide(), but every control word is read up front -- the whole first
+// Ctl line and the pull selector in one round trip, the bucket's ring word and the next
+// eight ring slots in a second -- instead of one dependent volatile load after another
+// (the general path's step cost ~4 us per bucket on C4, profiles/r02). Returns false
+// (nothing written) when the general path is needed: adaptive Delta, a heavy relaxation
+// that landed back in the bucket (reopen), or no non-empty slot among the next eight.
+__device__ bool decide_close_fast(const Params& p) {
+  volatile Ctl* c = p.ctl;
+  volatile SlotCtl* sc = p.sc;
+  u32 W[36];
+#pragma unroll
+  for (int i = 0; i < 9; ++i) {
+    const uint4 x = ld_volatile_v4(reinterpret_cast<const uint4*>(const_cast<Ctl*>(p.ctl)) + i);
+    W[4 * i] = x.x;
+    W[4 * i + 1] = x.y;
+    W[4 * i + 2] = x.z;
+    W[4 * i + 3] = x.w;
+  }
+  static_assert(offsetof(Ctl, cur) == 0 && offsetof(Ctl, lim) == 4 && offsetof(Ctl, mode) == 8 &&
+                offsetof(Ctl, far_min) == 12 && offsetof(Ctl, p2_end) == 20 && offsetof(Ctl, epochs) == 28 &&
+                offsetof(Ctl, cur_end) == 64 && offsetof(Ctl, a_mode) == 68 && offsetof(Ctl, a_m) == 108 &&
+                offsetof(Ctl, csum) == 116 && offsetof(Ctl, pull_sel) == 128, "Ctl layout (decide_close_fast)");
+  const u32 cur = W[0], lim0 = W[1], mode = W[2], fm = W[3], p2_end = W[5], epochs = W[7];
+  const u32 cur_end = W[16], a_mode = W[17], a_m = W[27], csum = W[29], pull_sel = W[32];
+  if (a_mode) return false;
+  const u32 s = cur & p.kmask;
+  const u64 ws = sc[s].word;
+  u32 t[8];
+#pragma unroll
+  for (u32 k = 0; k < 8; ++k)
+    t[k] = (cur_end + k <= lim0 && cur_end + k >= cur_end) ? (u32)(sc[(cur_end + k) & p.kmask].word >> 32) : 0u;
+  if ((u32)ws != 0) return false;  // reopen (f32 rounding): general path
+  u32 nxt = NONE, nxt_tail = 0;
+#pragma unroll
+  for (u32 k = 0; k < 8; ++k)
+    if (t[k] && nxt == NONE) {
+      nxt = cur_end + k;
+      nxt_tail = t[k];
+    }
+  if (nxt == NONE && cur_end + 8 <= lim0 && cur_end + 8 > cur_end) return false;  // scan further: general path
+  sc[s].p2 = p2_end;
+  if (mode == MODE_PULL || mode == MODE_PULL_LONG) c->pull_sel = pull_sel == 0 ? 1u : 0u;  // its output list
+  c->csum = 0;
+  c->closed_c = (p.claim_max & LOCAL_CHASE) ? NONE : csum;
+  c->closed_b = cur;
+  if (nxt == NONE && fm == NONE) {
+    c->mode = MODE_DONE;
+    return true;
+  }
+  if (fm <= nxt) {  // a dropped push precedes the ring's next bucket
+    c->rescan_base = fm;
+    c->mode = MODE_RESCAN_CLEAR;
+    return true;
+  }
+  sc[s].word = 0;  // recycle the finished bucket's queue (entries already SENTINEL)
+  sc[s].head = 0;
+  sc[s].p2 = 0;
+  const u32 lim = (u32)min((u64)nxt + p.K - 1, (u64)NONE - 1);  // see decide(): slots hold [nxt, nxt + K)
+  c->lim = lim;
+  c->cur = nxt;
+  c->cur_end = (u32)min((u64)nxt + a_m, (u64)lim + 1);
+  c->epochs = epochs + 1;
+  c->round_end = min(nxt_tail, p.cap);
+  c->mode = MODE_PHASE1;
+  return true;
+}
+
 // Last CTA to arrive runs the serial scheduler step (fused phase 3).
 __device__ void decide(const Params& p, u32 which) {
   volatile Ctl* c = p.ctl;
@@ -1155,6 +1232,8 @@ __device__ void decide(const Params& p, u32 which) {
     c->hub_word = (u64)(tail - b);  // pending = static entries; chunks add to it
     c->hub_head = 0;
     c->mode = MODE_PHASE2;
+  } else if (which == SYNC_P2 && decide_close_fast(p)) {
+    // fixed Delta: done with two round trips of loads (decide_close_fast)
   } else if (which == SYNC_P2) {
     const u32 cur = c->cur, s = cur & p.kmask;
     sc[s].p2 = c->p2_end;
@@ -1361,9 +1440,18 @@ __device__ void phase1(const Params& p, Smem& sm) {
         n = h < re ? min(c, re - h) : 0u;
       }
       for (; !loc && !(ABL && (p.flags & 2u));) {
-        const u64 wv = ld_relaxed_u64(&sc->word);
-        const u32 tail = min((u32)(wv >> 32), p.cap);
-        if (my_next >= my_end && my_end < p.cap) {
+        // word (tail, pend) and the ticket head in one 16-byte load (same control line)
+        uint4 cl;
+        asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(cl.x), "=r"(cl.y), "=r"(cl.z), "=r"(cl.w)
+                     : "l"(sc)
+                     : "memory");
+        const u64 wv = ((u64)cl.y << 32) | cl.x;
+        const u32 tail = min(cl.y, p.cap);
+        // Take new tickets only while some entry is unclaimed (head < tail): in a near-empty
+        // bucket the whole grid no longer queues 592 atomics on the one head word before the
+        // few CTAs that get entries can start (tickets past the tail still fill as pushes land).
+        if (my_next >= my_end && my_end < p.cap && cl.z < tail) {
           // claim size grows with the queue: small early (spread work), up to claim_max
           u32 c = min(max(tail / (2 * G), 8u), claim_max);
           my_next = atomicAdd(&sc->head, c);

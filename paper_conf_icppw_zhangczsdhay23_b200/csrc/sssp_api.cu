@@ -97,7 +97,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP, p_bdiv = 1;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP;
   i64 hub_ids_cached = -1;
   int sym_state = -1;  // arc multiset symmetric? -1 unknown (checked on demand after a weight sort)
   i64 v_nz = -1;       // degree-sorted graphs: vertices with arcs are ids [0, v_nz); -1 unknown
@@ -351,10 +351,6 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
       if (v < 1 || v > (i64)LOC_CAP) return fail(SSSP_ERR_INVALID_ARGUMENT, "local limit in [1,%u]", LOC_CAP);
       g->p_local_lim = v;
       return SSSP_OK;
-    case SSSP_PARAM_BUCKET_DIV:
-      if (v < 1 || v > 16) return fail(SSSP_ERR_INVALID_ARGUMENT, "bucket div in [1,16]");
-      g->p_bdiv = v;
-      return SSSP_OK;
     case SSSP_PARAM_CLAIM_MAX:
       if (v < 1 || v > (i64)BATCH) return fail(SSSP_ERR_INVALID_ARGUMENT, "claim max in [1,%u]", BATCH);
       g->p_claim = v;
@@ -602,16 +598,6 @@ static void adapt_params(sssp_graph_t g, int mode, DeltaParams* dp) {
   dp->ai = AdaptInit{(u32)mode, (float)d0, m0, mmin, mmax, l, 0u};
 }
 
-// SSSP_PARAM_BUCKET_DIV (u32, fixed Delta): buckets of width W = Delta / div while light
-// stays w < Delta. Delta-stepping's correctness needs only heavy arcs (relaxed once, after
-// their bucket) to be >= the bucket width, which w >= Delta >= W gives; light arcs may now
-// also push into the next bucket(s). Same distances; a schedule experiment.
-static void bucket_div(sssp_graph_t g, DeltaParams* dp) {
-  if (g->p_bdiv <= 1 || g->wtype != SSSP_WEIGHT_U32 || dp->ai.mode || dp->delta_u == 0xFFFFFFFFu) return;
-  dp->delta_u = std::max<u32>(1u, dp->delta_u / (u32)g->p_bdiv);
-  dp->ahead = (double)g->maxw_bits / dp->delta_u;
-}
-
 static sssp_status delta_params(sssp_graph_t g, double delta, DeltaParams* dp) {
   dp->ai = AdaptInit{0u, 1.f, 1u, 1u, 1u, 0u, 0u};
   if (std::isnan(delta) || delta <= 0.0) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta must be > 0 (got %g)", delta);
@@ -857,7 +843,6 @@ extern "C" sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta) {
   DeltaParams dp;
   if ((st = delta_params(g, delta, &dp))) return st;
   adapt_params(g, (int)g->p_adapt, &dp);
-  bucket_div(g, &dp);
   DeviceGuard dg(g->device);
   const u32 src = g->h_old2new.empty() ? (u32)source : g->h_old2new[source];
   g->have_result = false;
@@ -972,7 +957,6 @@ extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, in
   DeltaParams dp;
   if ((st = delta_params(g, delta, &dp))) return st;
   adapt_params(g, (int)g->p_adapt, &dp);
-  bucket_div(g, &dp);
   for (i64 i = 0; i < n; ++i)
     if (sources[i] < 0 || sources[i] >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source[%lld] out of range", (long long)i);
   DeviceGuard dg(g->device);

@@ -882,28 +882,3 @@ def test_pull_symmetric_is_checked(sssp):
     with sssp.Graph(row, col, w) as G:
         G.reorder()
         assert G.is_symmetric()
-
-
-@pytest.mark.parametrize("div", [2, 4])
-def test_bucket_div_parity(sssp, div):
-    """SSSP_PARAM_BUCKET_DIV: buckets of width Delta/div, light still w < Delta (heavy arcs
-    w >= Delta >= width land in later buckets): bit-exact distances on Kronecker graphs with
-    pull on and off and on a grid; bucket counts then follow the narrower width."""
-    for g, deltas in ((gen.kronecker(13, 16, seed=51), (8, 16, 64)), (gen.grid(300, 200, p=0.2, seed=5), (400, 1600))):
-        srcs = [int(x) for x in gen.sample_sources(g, 2, seed=2)]
-        exp = {s: oracle.dijkstra(g.row, g.col, g.w, s) for s in srcs}
-        for pull in (1, 0):
-            with sssp.Graph(g.row, g.col, g.w) as G:
-                G.reorder()
-                G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, pull)
-                G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, 0)
-                G.set_param(sssp.SSSP_PARAM_BUCKET_DIV, div)
-                for d in deltas:
-                    for s in srcs:
-                        assert_same(G.sssp(s, d), exp[s], f"div={div} pull={pull} V={g.V} delta={d} src={s}")
-                        w = max(1, int(math.ceil(d)) // div)
-                        closed = {b: c for b, _, c in _closed_buckets(G.trace())}
-                        hist = oracle.bucket_histogram(exp[s], w)
-                        for b in range(len(hist)):
-                            if hist[b]:
-                                assert closed.get(b) == int(hist[b]), f"div={div} delta={d} bucket {b}"

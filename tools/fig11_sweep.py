@@ -8,7 +8,11 @@ the mean over N seeded sources at the best Delta, persistent-kernel time
 from CUDA events (sssp_kernel_time). Prints one line per graph plus the
 paper's V100 number.
 
-python tools/fig11_sweep.py [--scales 22 23 24] [--efs 8 16 32 64] [--sources 16]
+--directed: one arc per generated edge (reading R13: the paper's s24 ef64 would not fit
+its 16 GB V100 symmetrised, P:1186), push phases 2&3 (the pull needs symmetry);
+otherwise symmetrised with the pull phases 2&3 (SSSP_PARAM_PULL_SYMMETRIC, verified).
+
+python tools/fig11_sweep.py [--scales 22 23 24] [--efs 8 16 32 64] [--sources 16] [--directed]
 """
 import argparse
 import os
@@ -34,21 +38,27 @@ def main():
     ap.add_argument("--deltas", type=float, nargs="*", default=[80, 160, 320])
     ap.add_argument("--sources", type=int, default=16)
     ap.add_argument("--seed", type=int, default=11)
+    ap.add_argument("--directed", action="store_true")
+    ap.add_argument("--no-pull", action="store_true")
     a = ap.parse_args()
     import torch  # noqa: F401  (CUDA context, device memory)
 
     import paper_conf_icppw_zhangczsdhay23_b200 as sssp
 
+    print(f"# storage: {'directed (one arc per edge)' if a.directed else 'symmetrised'}, "
+          f"phases 2&3: {'push' if a.directed or a.no_pull else 'pull for large buckets'}", flush=True)
     print("scale ef  V          arcs        best_delta  ms/SSSP  GTEPS   paper_V100  ratio  gen_s  reorder_ms", flush=True)
     for s in a.scales:
         for ef in a.efs:
             t0 = time.time()
-            g = gen.kronecker(s, ef, seed=a.seed, weights="u32", lo=1, hi=1000)
+            g = gen.kronecker(s, ef, seed=a.seed, weights="u32", lo=1, hi=1000, symmetrize=not a.directed)
             gen_s = time.time() - t0
             srcs = gen.sample_sources(g, a.sources, seed=7)
             with sssp.Graph(g.row, g.col, g.w, device=0) as G:
                 G.reorder()
                 reorder_ms = G.stats()["reorder_ms"]
+                if not a.directed and not a.no_pull:
+                    G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
                 best = None
                 for d in a.deltas:
                     G.run(int(srcs[0]), d)  # warm-up (heavy offsets for this Delta)

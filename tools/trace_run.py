@@ -11,7 +11,7 @@ import numpy as np  # noqa: E402
 
 import gen  # noqa: E402
 
-NAMES = {0: "P1", 1: "P2", 2: "RC", 3: "RF", 4: "SL", 5: "SH", 6: "P2C", 7: "MG", 9: "PL", 99: "start"}
+NAMES = {0: "P1", 1: "P2", 2: "RC", 3: "RF", 4: "SL", 5: "SH", 6: "P2C", 7: "MG", 8: "ADAPT", 9: "PL", 10: "F", 99: "start"}
 
 
 def main():
