@@ -61,6 +61,9 @@ constexpr u32 HUB_CHUNK = 4096;
 #ifndef SSSP_DEFER_ATOMICS
 #define SSSP_DEFER_ATOMICS 1  // relaxations' atomicMin issued by pb_flush, a staged batch at once
 #endif
+#ifndef SSSP_STATIC_TASKS
+#define SSSP_STATIC_TASKS 1  // batch tasks dealt round-robin to the warps (no shared-memory claim atomic)
+#endif
 #ifndef SSSP_BATCH_SAMPLES
 #define SSSP_BATCH_SAMPLES 0  // per-batch stage/task/tail cycles in sssp_get_samples (diagnostics build)
 #endif
@@ -284,6 +287,7 @@ struct Smem {
   u32 fc[DS_WARPS][64];      // pb_flush: entries per ring slot, then each slot's next position
   FlushCtx fctx;
   unsigned long long st[ST_N];
+  unsigned long long wst[DS_WARPS][ST_N];  // per-warp counters (st_add), summed at kernel end
   u32 claim_h, claim_n, claim_src;
   // CTA-local chase (LOCAL_CHASE): phase-1 pushes into the current bucket kept in shared
   // memory and processed by this CTA next, without the global queue round trip
@@ -374,7 +378,7 @@ __device__ __forceinline__ u32 bucket_of(const Params& p, u32 d) {
 
 __device__ __forceinline__ void st_add(Smem& sm, int k, u32 x) {
   u32 s = __reduce_add_sync(SSSP_FULL_MASK, x);
-  if (lane_id() == 0 && s) atomicAdd(&sm.st[k], (unsigned long long)s);
+  if (lane_id() == 0 && s) sm.wst[threadIdx.x >> 5][k] += s;  // this warp's row: no atomic
 }
 
 // Publish warp w's staged pushes: per 32 entries, one global reservation per
@@ -439,7 +443,7 @@ __device__ __noinline__ void pb_flush_impl(Smem& sm, u32 lim, u32 nearb) {
       }
     }
     nsurv = __reduce_add_sync(SSSP_FULL_MASK, nsurv);
-    if (lane == 0) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)nsurv);
+    if (lane == 0) sm.wst[w][ST_UPDATES] += nsurv;
     __syncwarp();
   }
   const u32 c0 = sm.cur, ce = sm.cur_end;
@@ -928,6 +932,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   const u32 ntask = S + sm.rl_tasks, nl = sm.rl_n;
   if (tid == 0) sm.st[ST_P_NT] += ntask;
   // Task descriptor -> per-lane arc indices / distances (smem lookups only).
+  u32 rl_cur = 0;  // SSSP_STATIC_TASKS: this warp's current range-list entry
   auto setup = [&](u32 t, u32 (&idx)[UNROLL], bool (&valid)[UNROLL], u32 (&dd)[UNROLL]) {
     if (t >= ntask) {
 #pragma unroll
@@ -954,6 +959,12 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       }
     } else {  // range-list slice
       const u32 tr = t - S;
+#if SSSP_STATIC_TASKS
+      // a warp's tasks ascend by DS_WARPS: walk on from its previous entry
+      u32 lo = rl_cur;
+      while (lo + 1 < nl && sm.rl_toff[lo + 1] <= tr) ++lo;
+      rl_cur = lo;
+#else
       u32 lo = 0, hi = nl;  // entry i with toff[i] <= tr < toff[i+1]
       while (hi - lo > 1) {
         const u32 mid = (lo + hi) >> 1;
@@ -962,6 +973,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
         else
           hi = mid;
       }
+#endif
       const u32 sub = (tr - sm.rl_toff[lo]) * TASK;
       const u32 b = sm.rl_beg[lo] + sub;
       const u32 l = sm.rl_len[lo] - sub;
@@ -975,11 +987,20 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       }
     }
   };
+#if SSSP_STATIC_TASKS
+  u32 t_next = w;  // round-robin: tasks cost about the same (<= 64 arcs, latency-bound)
+  auto claim = [&]() {
+    const u32 t = t_next;
+    t_next += DS_WARPS;
+    return t;
+  };
+#else
   auto claim = [&]() {
     u32 t = 0;
     if (lane == 0) t = atomicAdd(&sm.task_next, 1u);
     return __shfl_sync(SSSP_FULL_MASK, t, 0);
   };
+#endif
   u32 idx[UNROLL], dd[UNROLL];
   bool valid[UNROLL];
   uint2 a[UNROLL];
@@ -2210,7 +2231,7 @@ __device__ void merge_slots(const Params& p, Smem& sm) {
   }
   if (sm.pb_n[threadIdx.x >> 5]) pb_flush<F32>(p, sm, lim, NONE);
   const u32 mv = __reduce_add_sync(SSSP_FULL_MASK, moved);
-  if (lane == 0 && mv) atomicAdd(&sm.st[ST_UPDATES], (unsigned long long)(-(long long)mv));  // not updates
+  if (lane == 0 && mv) sm.wst[threadIdx.x >> 5][ST_UPDATES] -= mv;  // not updates
 }
 
 // ABL = extended build: the ablation paths (SSSP_PARAM_ADWL = 0 / SSSP_PARAM_SYNC = 1),
@@ -2227,6 +2248,7 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     p.ctl->trace_n = 1;
   }
   if (threadIdx.x < ST_N) sm.st[threadIdx.x] = 0;
+  for (u32 i = threadIdx.x; i < DS_WARPS * ST_N; i += blockDim.x) (&sm.wst[0][0])[i] = 0;
   if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
     sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.dist, p.cap, p.kmask, p.delta_u, p.inv_delta};
@@ -2282,7 +2304,12 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     }
   }
   __syncthreads();
-  if (threadIdx.x < ST_N && sm.st[threadIdx.x]) atomicAdd(p.stats + threadIdx.x, sm.st[threadIdx.x]);
+  if (threadIdx.x < ST_N) {
+    unsigned long long x = sm.st[threadIdx.x];
+#pragma unroll
+    for (int w = 0; w < DS_WARPS; ++w) x += sm.wst[w][threadIdx.x];
+    if (x) atomicAdd(p.stats + threadIdx.x, x);
+  }
   // Every CTA has passed the last grid barrier, so err is final: fold it into the sticky word
   // that sssp_wait / sssp_run_batch / sssp_distances report (and clear) on the host.
   if (blockIdx.x == 0 && threadIdx.x == 0) {
