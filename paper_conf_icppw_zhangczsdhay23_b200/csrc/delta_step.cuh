@@ -259,6 +259,7 @@ struct FlushCtx {
   Ctl* ctl;
   u32* xd;
   u32* dist;
+  u64 dmul;  // u32 graphs: ceil(2^64 / delta_u), so d / delta_u = umulhi64(d, dmul) exactly
   u32 cap, kmask, delta_u;
   float inv_delta;
 };
@@ -392,7 +393,9 @@ __device__ __forceinline__ u32 bucket_of_f(const FlushCtx& p, u32 d) {
     u32 b = __float2uint_rz(__fmul_rn(__uint_as_float(d), p.inv_delta));
     return b >= NONE ? NONE - 1 : b;
   } else {
-    return d / p.delta_u;
+    // floor(d / delta_u) as a 64-bit multiply-high: with dmul = ceil(2^64 / D) the error is
+    // below d / 2^64 < 2^-32, less than the gap between d / D and the next integer
+    return p.delta_u == 1 ? d : (u32)__umul64hi((u64)d, p.dmul);
   }
 }
 
@@ -698,20 +701,6 @@ __device__ __forceinline__ void relax_finish(const Params& p, Smem& sm, u32 lim,
 #endif
 }
 
-// Range of an item for phase PH: PRO -> light [start, heavy) / heavy [heavy, end);
-// no PRO -> the whole adjacency (predicate per arc).
-template <bool PRO, int PH, bool EXT>
-__device__ __forceinline__ void item_range(const Params& p, const Smem& sm, u32 v, i64& b, i64& e) {
-  const uint2* rowc = EXT ? p.rowc + sm.rowc_off : p.rowc;  // heavy offsets of the bucket's level
-  const uint2 r = rowc[v];
-  if (PRO && PH == 1) {
-    b = r.x;
-    e = r.y;
-  } else {
-    e = rowc[v + 1].x;
-    b = (PRO && PH == 2) ? r.y : r.x;
-  }
-}
 
 // ------------------------------------------------------------ batch -------
 // Batch item q (0 <= q < n) lives in thread (x % 8) * 32 + x / 8 of round
@@ -744,6 +733,21 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
     cls[i] = 0;
     cd[i] = has[i] ? ld_cg(p.dist + (lo & ~CHUNK_FLAG)) : 0u;
   }
+  // item range for phase PH: PRO -> light [start, heavy) / heavy [heavy, end); no PRO -> the
+  // whole adjacency (predicate per arc). (Loading the rows with the dist probe, for stale
+  // entries too, measured 4 % slower on C4.)
+  const uint2* rowc = EXT ? p.rowc + sm.rowc_off : p.rowc;  // heavy offsets of the bucket's level
+  auto range_of = [&](int i, i64& b, i64& e) {
+    const u32 v = (u32)it[i] & ~CHUNK_FLAG;
+    const uint2 r = rowc[v];
+    if (PRO && PH == 1) {
+      b = r.x;
+      e = r.y;
+    } else {
+      e = rowc[v + 1].x;
+      b = (PRO && PH == 2) ? r.y : r.x;
+    }
+  };
   u32 c_settled = 0, c_stale = 0, c_arcs = 0, c_chunks = 0, c_w = 0, c_c = 0, c_t = 0;
 #pragma unroll
   for (int i = 0; i < N; ++i) {
@@ -758,7 +762,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       // Chunk items in the phase-2 static range are phase-1 work already done.
       if (!(PH == 2 && src == SRC_STATIC)) {
         i64 rb, re;
-        item_range<PRO, PH, EXT>(p, sm, v, rb, re);
+        range_of(i, rb, re);
         const i64 b = rb + (i64)hi * HUB_CHUNK;
         beg[i] = (u32)b;
         len[i] = (u32)min((i64)HUB_CHUNK, re - b);
@@ -774,7 +778,7 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
       } else {
         c_settled += 1;
         i64 rb, re;
-        item_range<PRO, PH, EXT>(p, sm, v, rb, re);
+        range_of(i, rb, re);
         const i64 l = re - rb;
         if (!ADWL) {  // ablation: the vertex's own thread walks all its arcs
           beg[i] = (u32)rb;
@@ -1500,7 +1504,7 @@ __device__ void phase1(const Params& p, Smem& sm) {
       sm.claim_h = h;
       sm.claim_src = loc;
       sm.st[ST_P_CLAIM] += (unsigned long long)(clock64() - t_c);
-      if (blockIdx.x % SAMPLE_EVERY == 0) {  // claim timeline (which = 100): tail / pend / ticket
+      if (SSSP_BATCH_SAMPLES && blockIdx.x % SAMPLE_EVERY == 0) {  // claim timeline (which = 100)
         const u32 k = atomicAdd(&p.ctl->sample_n, 1u);
         if (k < SAMPLE_CAP) {
           const u64 wv = ld_relaxed_u64(&sc->word);
@@ -2251,7 +2255,9 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
   for (u32 i = threadIdx.x; i < DS_WARPS * ST_N; i += blockDim.x) (&sm.wst[0][0])[i] = 0;
   if (threadIdx.x < DS_WARPS) sm.pb_n[threadIdx.x] = 0;
   if (threadIdx.x == 0) {
-    sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.dist, p.cap, p.kmask, p.delta_u, p.inv_delta};
+    // dmul = ceil(2^64 / delta_u); delta_u = 1 (2^64 does not fit) is its own case in bucket_of_f
+    const u64 dm = p.delta_u > 1 ? (~0ULL / p.delta_u) + 1 : 0ULL;
+    sm.fctx = FlushCtx{p.sc, p.items, p.ctl, p.xd, p.dist, dm, p.cap, p.kmask, p.delta_u, p.inv_delta};
     sm.loc_n = 0;
     sm.loc_on = 0;
     volatile Ctl* vc = p.ctl;
