@@ -509,29 +509,44 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
     // chunks over all blocks. The hub count is bounded by A / EXPAND_HUB, so
     // the chunk scan runs over that capacity with no host round trip.
     CT(cudaMemsetAsync(hubs + nh_cap, 0, sizeof(u32), s));
+    // (src', w, dst') as one 64-bit key when src', w and dst' fit (S = w's end rounded up to
+    // whole 8-bit digits): each radix pass then moves 8 bytes per arc instead of 12
+    const int vb = std::max(1, bits_for((u64)(V - 1))), wb = bits_for(g->maxw_bits);
+    const int S = (vb + wb + 7) / 8 * 8;
+    ArcPack pk{(S + vb <= 64) ? 1 : 0, vb, S};
     k_list_hubs<<<grid_for(V), 256, 0, s>>>(g->rowp, V, hubs, hubs + nh_cap);
     k_expand_arcs_flat<<<grid_for(V), 256, 0, s>>>(g->rowp, g->arcs, V, deg ? g->old2new : nullptr,
-                                                   f[0], f[1], f[2]);
+                                                   f[0], f[1], f[2], pk);
     k_hub_chunks<<<(nh_cap + 256) / 256, 256, 0, s>>>(g->rowp, hubs, hubs + nh_cap, nh_cap, cst);
     scan_exclusive_rec<u32>(cst, cst, (i64)nh_cap + 1, ctmp, s);
     k_expand_hubs<<<g->num_sms * 8, 256, 0, s>>>(g->rowp, g->arcs, hubs, nh_cap, cst,
-                                                 deg ? g->old2new : nullptr, f[0], f[1], f[2]);
+                                                 deg ? g->old2new : nullptr, f[0], f[1], f[2], pk);
     CT(cudaGetLastError());
-    Fields<3> a{{f[0], f[1], f[2]}}, b{{f[3], f[4], f[5]}};
-    const int vb = bits_for((u64)(V - 1));
-    auto pass3 = [&](int kf, int sh) { return radix_pass<3>(g, a, b, kf, A, sh, hist, tmp); };
-    if (wsort) {
-      for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(2, sh);
-      const int wb = bits_for(g->maxw_bits);
-      for (int sh = 0; sh < wb && !st; sh += 8) st = pass3(1, sh);
+    if (pk.packed) {
+      // LSD over the key's digits: (w, dst') when weight-sorting, then src' (stable)
+      Fields<2> a{{f[0], f[1]}}, b{{f[3], f[4]}};
+      const int from = wsort ? 0 : S;
+      for (int sh = from; sh < S + vb && !st; sh += 8) st = radix_pass<2>(g, a, b, sh >= 32 ? 1 : 0, A, sh & 31, hist, tmp);
+      if (st) {
+        free_all();
+        return st;
+      }
+      k_unpack_sorted<<<grid_for(A), 256, 0, s>>>(a.f[0], a.f[1], A, pk, g->arcs);
+    } else {
+      Fields<3> a{{f[0], f[1], f[2]}}, b{{f[3], f[4], f[5]}};
+      auto pass3 = [&](int kf, int sh) { return radix_pass<3>(g, a, b, kf, A, sh, hist, tmp); };
+      if (wsort) {
+        for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(2, sh);
+        for (int sh = 0; sh < wb && !st; sh += 8) st = pass3(1, sh);
+      }
+      if (deg || wsort)
+        for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(0, sh);
+      if (st) {
+        free_all();
+        return st;
+      }
+      k_pack_sorted<<<grid_for(A), 256, 0, s>>>(a.f[1], a.f[2], A, g->arcs);
     }
-    if (deg || wsort)
-      for (int sh = 0; sh < vb && !st; sh += 8) st = pass3(0, sh);
-    if (st) {
-      free_all();
-      return st;
-    }
-    k_pack_sorted<<<grid_for(A), 256, 0, s>>>(a.f[1], a.f[2], A, g->arcs);
     CT(cudaGetLastError());
   }
   if (deg) k_set_rowp<<<grid_for(V + 1), 256, 0, s>>>(ndeg, V, A, g->rowp);
