@@ -242,7 +242,7 @@ typedef enum {
     SSSP_PARAM_PULL_SYMMETRIC = 11, /* 1 = the caller asserts the graph is symmetric (every arc
                                       (u,v,w) has its reverse (v,u,w), as the generators' graphs
                                       are, R13): graphs after a weight-sorting sssp_reorder
-                                      then run phases 2&3 of buckets holding >= V/16 entries as a
+                                      then run phases 2&3 of buckets holding >= V/128 entries as a
                                       pull (each unsettled vertex scans its weight-sorted heavy
                                       arcs up to the first that cannot win). Same distances.
                                       The assertion is verified once per reorder (sssp_is_

@@ -78,7 +78,7 @@ constexpr int IPT = SSSP_IPT;
 constexpr int IPT2 = SSSP_IPT2;
 constexpr int IPT_MAX = IPT > IPT2 ? IPT : IPT2;
 #ifndef SSSP_PULL_DIV
-#define SSSP_PULL_DIV 16u  // pull phase 2 when a bucket holds >= V / 16 entries
+#define SSSP_PULL_DIV 128u  // pull phases 2&3 when a bucket holds >= V / 128 entries (A/B on C4, C3: 128 beats 8-64, = 256; profiles/r02/ab_pull_div.txt)
 #endif
 #ifndef SSSP_CLAIM_MINPART
 #define SSSP_CLAIM_MINPART 64u  // take a partial batch once this many entries are ready ...

@@ -383,30 +383,38 @@ __device__ void ms_bucket_run(const MParams& p, MSmem& sm) {
     n = __shfl_sync(SSSP_FULL_MASK, n, 0);
     h = __shfl_sync(SSSP_FULL_MASK, h, 0);
     if (n == 0) break;
-    for (u32 i = 0; i < n; ++i) {
-      u64 e = SENTINEL;
-      if (lane == 0) {
-        u32 ns = 16;
-        while ((e = ld_relaxed_u64(q + h + i)) == SENTINEL) {  // reserved, not yet written
-          __nanosleep(ns);
-          if (ns < 256) ns <<= 1;
-        }
-        st_relaxed_u64(q + h + i, SENTINEL);
+    // Prologue of the whole claim at once (lane i: item i): wait for the entry, recycle it,
+    // read its arc range and take Q[v] -- one round trip of each for up to MS_CLAIM items
+    // instead of per item (the items are then relaxed one after another).
+    static_assert(MS_CLAIM <= 32, "one lane per claimed item");
+    u32 iv = 0, ib = 0, ie = 0, ix = NONE, ich = 0;
+    if (lane < n) {
+      u64 e;
+      u32 ns = 16;
+      while ((e = ld_relaxed_u64(q + h + lane)) == SENTINEL) {  // reserved, not yet written
+        __nanosleep(ns);
+        if (ns < 256) ns <<= 1;
       }
-      e = __shfl_sync(SSSP_FULL_MASK, e, 0);
-      const u32 lo = (u32)e, v = lo & ~CHUNK_FLAG;
-      u32 b = p.rowc[v].x, en = p.rowc[v + 1].x;
-      if (lo & CHUNK_FLAG) {
-        b += (u32)(e >> 32) * MS_CHUNK;
-        en = min(en, b + MS_CHUNK);
+      st_relaxed_u64(q + h + lane, SENTINEL);
+      const u32 lo = (u32)e;
+      iv = lo & ~CHUNK_FLAG;
+      ich = (lo & CHUNK_FLAG) ? 1u : 0u;
+      ib = p.rowc[iv].x;
+      ie = p.rowc[iv + 1].x;
+      if (ich) {
+        ib += (u32)(e >> 32) * MS_CHUNK;
+        ie = min(ie, ib + MS_CHUNK);
       } else {
-        u32 x = 0;
-        if (lane == 0) {
-          x = ms_q_take_acquire(p.Q + v);
-        }
-        x = __shfl_sync(SSSP_FULL_MASK, x, 0);
-        __syncwarp();
-        if (x == NONE) {  // already expanded through another entry
+        ix = ms_q_take_acquire(p.Q + iv);  // NONE: already expanded through another entry
+      }
+    }
+    __syncwarp();  // every take precedes the row reads below (acquire, then warp order)
+    for (u32 i = 0; i < n; ++i) {
+      const u32 v = __shfl_sync(SSSP_FULL_MASK, iv, i);
+      const u32 b = __shfl_sync(SSSP_FULL_MASK, ib, i), en = __shfl_sync(SSSP_FULL_MASK, ie, i);
+      const u32 x = __shfl_sync(SSSP_FULL_MASK, ix, i), ch = __shfl_sync(SSSP_FULL_MASK, ich, i);
+      if (!ch) {
+        if (x == NONE) {
           ++c_stale;
           continue;
         }
