@@ -2,6 +2,7 @@
 // Host side: validation, device memory, stream-ordered launches. Every step
 // of the SSSP path runs in the kernels of pro.cuh / sort.cuh / delta_step.cuh.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges cost nothing without a profiler
 
 #include <algorithm>
 #include <cmath>
@@ -19,6 +20,12 @@
 #include "sort.cuh"
 
 using namespace sssp;
+
+// NVTX range over one ABI call (visible in Nsight Systems / ncu --nvtx).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 // --------------------------------------------------------------- errors ---
 static thread_local std::string g_last_error;
@@ -142,6 +149,7 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
                                          const int64_t* row, const uint32_t* col,
                                          const void* weights, sssp_weight_type wtype,
                                          sssp_memory where, void* cuda_stream) {
+  NvtxRange nvtx_("sssp_graph_create");
   sssp_graph_s* g = nullptr;
   if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
   if (V < 1 || V >= 0x7FFFFFFFLL) return fail(SSSP_ERR_INVALID_ARGUMENT, "V=%lld out of [1, 2^31-1)", (long long)V);
@@ -361,6 +369,7 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
 
 // ------------------------------------------------------------- symmetry --
 extern "C" sssp_status sssp_is_symmetric(sssp_graph_t g, int* out) {
+  NvtxRange nvtx_("sssp_is_symmetric");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
@@ -414,6 +423,7 @@ static int bits_for(u64 maxv) {
 }
 
 extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
+  NvtxRange nvtx_("sssp_reorder");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (flags & ~(SSSP_PRO_DEGREE | SSSP_PRO_WEIGHT)) return fail(SSSP_ERR_INVALID_ARGUMENT, "bad PRO flags 0x%x", flags);
@@ -852,6 +862,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
 }
 
 extern "C" sssp_status sssp_run(sssp_graph_t g, int64_t source, double delta) {
+  NvtxRange nvtx_("sssp_run");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (source < 0 || source >= g->V) return fail(SSSP_ERR_INVALID_ARGUMENT, "source %lld out of range", (long long)source);
@@ -885,6 +896,7 @@ static sssp_status take_run_errors(sssp_graph_t g) {
 }
 
 extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory where) {
+  NvtxRange nvtx_("sssp_distances");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
@@ -916,6 +928,7 @@ extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory whe
 }
 
 extern "C" sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memory where) {
+  NvtxRange nvtx_("sssp_distances_async");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
@@ -955,6 +968,7 @@ extern "C" sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memo
 }
 
 extern "C" sssp_status sssp_wait(sssp_graph_t g) {
+  NvtxRange nvtx_("sssp_wait");
   sssp_status st = check_handle(g);
   if (st) return st;
   DeviceGuard dg(g->device);
@@ -965,6 +979,7 @@ extern "C" sssp_status sssp_wait(sssp_graph_t g) {
 
 extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                                       void* out_dev, int64_t ld) {
+  NvtxRange nvtx_("sssp_run_batch");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (n < 0 || (n > 0 && (!sources || !out_dev)) || ld < g->V)
@@ -990,6 +1005,7 @@ extern "C" sssp_status sssp_run_batch(sssp_graph_t g, const int64_t* sources, in
 // NEXT-4: up to 32 sources per persistent launch (multi_source.cuh).
 extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, int64_t n, double delta,
                                       void* out_dev, int64_t ld) {
+  NvtxRange nvtx_("sssp_run_multi");
   sssp_status st = check_handle(g);
   if (st) return st;
   if (n < 0 || (n > 0 && (!sources || !out_dev)) || ld < g->V)
