@@ -24,6 +24,7 @@
 #ifndef SSSP_H
 #define SSSP_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -326,6 +327,20 @@ sssp_status sssp_get_profile(sssp_graph_t g, uint64_t* out, int n);
  * every run of equal arcs is matched by a lower_bound in the other end's
  * sorted segment (one kernel, cached until the next reorder). Synchronises. */
 sssp_status sssp_is_symmetric(sssp_graph_t g, int* out);
+
+/* Device-memory allocator hook (process-wide; "the library allocates device
+ * memory through an optional allocator hook, so torch's caching allocator can back it").
+ * With a hook set, every device buffer a handle owns (graph, queues, distances, staging,
+ * reorder temporaries) comes from alloc(bytes, device, stream, ctx), which returns NULL on
+ * failure (-> SSSP_ERR_OUT_OF_MEMORY), and goes back through the free_fn of the hook that
+ * made it (ptr, bytes, device, stream, ctx) -- also after the hook changes, so set it before
+ * creating handles for consistency. The library synchronises its stream before it frees a
+ * buffer that work may still use. NULL, NULL restores cudaMalloc / cudaFree; exactly one of
+ * the two NULL is SSSP_ERR_INVALID_ARGUMENT. Small per-call scratch words still use
+ * stream-ordered cudaMallocAsync. */
+typedef void* (*sssp_alloc_fn)(size_t bytes, int device, void* cuda_stream, void* ctx);
+typedef void (*sssp_free_fn)(void* ptr, size_t bytes, int device, void* cuda_stream, void* ctx);
+sssp_status sssp_set_allocator(sssp_alloc_fn alloc, sssp_free_fn free_fn, void* ctx);
 
 /* Library/device info: number of SMs of the handle's device. */
 int sssp_device_sm_count(sssp_graph_t g);

@@ -60,7 +60,7 @@ EXPORTS = (
     "sssp_destroy", "sssp_status_string", "sssp_last_error", "sssp_set_stream", "sssp_run_batch",
     "sssp_get_stats", "sssp_export_csr", "sssp_set_param", "sssp_device_sm_count",
     "sssp_kernel_time", "sssp_get_trace", "sssp_get_profile", "sssp_run_multi", "sssp_multi_stats",
-    "sssp_distances_async", "sssp_wait", "sssp_is_symmetric", "sssp_get_samples",
+    "sssp_distances_async", "sssp_wait", "sssp_is_symmetric", "sssp_get_samples", "sssp_set_allocator",
 )
 
 
@@ -93,6 +93,10 @@ _lib.sssp_run_multi.argtypes = [_P, _P, _I64, _D, _P, _I64]
 _lib.sssp_distances_async.argtypes = [_P, _P, _I]
 _lib.sssp_wait.argtypes = [_P]
 _lib.sssp_is_symmetric.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+_lib.sssp_set_allocator.argtypes = [_ALLOC_FN, _FREE_FN, _P]
+_lib.sssp_set_allocator.restype = ctypes.c_int
 _lib.sssp_multi_stats.argtypes = [_P, _P, _I64]
 _lib.sssp_get_stats.argtypes = [_P, ctypes.POINTER(sssp_stats)]
 _lib.sssp_export_csr.argtypes = [_P, _D, _P, _P, _P, _P]
@@ -309,6 +313,40 @@ def sssp_get_profile(h):
     out = np.zeros(len(names), dtype=np.uint64)
     _check(_lib.sssp_get_profile(h, out.ctypes.data, len(names)), "sssp_get_profile")
     return dict(zip(names, out.tolist()))
+
+
+_alloc_keep = None  # the ctypes callbacks must outlive every buffer they made
+
+
+def sssp_set_allocator(alloc=None, free=None):
+    """Route the library's device buffers through Python callables:
+    alloc(bytes, device, stream) -> int pointer (0 on failure); free(ptr, bytes, device, stream).
+    Both None restores cudaMalloc / cudaFree (buffers made by a hook still go back to it)."""
+    global _alloc_keep
+    if alloc is None and free is None:
+        _check(_lib.sssp_set_allocator(_ALLOC_FN(), _FREE_FN(), None), "sssp_set_allocator")
+        return
+    a = _ALLOC_FN(lambda n, dev, st, ctx: alloc(n, dev, st or 0) or None)
+    f = _FREE_FN(lambda ptr, n, dev, st, ctx: free(ptr, n, dev, st or 0))
+    _check(_lib.sssp_set_allocator(a, f, None), "sssp_set_allocator")
+    _alloc_keep = (_alloc_keep or []) + [(a, f)]
+
+
+def use_torch_allocator():
+    """Back the library's device memory with PyTorch's caching allocator (sssp.h
+    sssp_set_allocator): the buffers show up in torch.cuda.memory_allocated()."""
+    import torch
+
+    def alloc(n, dev, stream):
+        try:
+            return torch.cuda.caching_allocator_alloc(n, dev, stream if stream else None)
+        except RuntimeError:
+            return 0
+
+    def free(ptr, n, dev, stream):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    sssp_set_allocator(alloc, free)
 
 
 def sssp_is_symmetric(h):

@@ -6,6 +6,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <mutex>
+#include <unordered_map>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -26,6 +28,71 @@ struct NvtxRange {
   explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
   ~NvtxRange() { nvtxRangePop(); }
 };
+
+// ------------------------------------------------------ allocator hook ---
+// sssp_set_allocator: device buffers of every handle come from the hook (e.g. torch's caching
+// allocator) when one is set; each buffer remembers the hook that made it, so it is always
+// returned to the same one, also after the hook changes.
+struct AllocHook {
+  sssp_alloc_fn alloc = nullptr;
+  sssp_free_fn free = nullptr;
+  void* ctx = nullptr;
+};
+static std::mutex g_alloc_mu;
+static AllocHook g_hook;
+static std::unordered_map<void*, std::pair<AllocHook, size_t>> g_hooked;
+
+static cudaError_t dalloc(void** ptr, size_t bytes, cudaStream_t s = nullptr) {
+  AllocHook h;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    h = g_hook;
+  }
+  if (!h.alloc) return cudaMalloc(ptr, bytes);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  void* q = h.alloc(bytes, dev, (void*)s, h.ctx);
+  if (!q) return cudaErrorMemoryAllocation;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    g_hooked[q] = {h, bytes};
+  }
+  *ptr = q;
+  return cudaSuccess;
+}
+template <class T>
+static cudaError_t dalloc(T** ptr, size_t bytes, cudaStream_t s = nullptr) {
+  return dalloc(reinterpret_cast<void**>(ptr), bytes, s);
+}
+
+static cudaError_t dfree(void* ptr, cudaStream_t s = nullptr) {
+  if (!ptr) return cudaSuccess;
+  AllocHook h;
+  size_t bytes = 0;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    auto it = g_hooked.find(ptr);
+    if (it != g_hooked.end()) {
+      h = it->second.first;
+      bytes = it->second.second;
+      g_hooked.erase(it);
+    }
+  }
+  if (!h.free) return cudaFree(ptr);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  h.free(ptr, bytes, dev, (void*)s, h.ctx);
+  return cudaSuccess;
+}
+
+extern "C" sssp_status sssp_set_allocator(sssp_alloc_fn alloc, sssp_free_fn free_fn, void* ctx) {
+  if ((alloc == nullptr) != (free_fn == nullptr)) return SSSP_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lk(g_alloc_mu);
+  g_hook.alloc = alloc;
+  g_hook.free = free_fn;
+  g_hook.ctx = ctx;
+  return SSSP_OK;
+}
 
 // --------------------------------------------------------------- errors ---
 static thread_local std::string g_last_error;
@@ -190,24 +257,24 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
         break;                                                                          \
       }                                                                                 \
     }
-    CG(cudaMalloc(&g->rowp, sizeof(longlong2) * (V + 1)));
-    CG(cudaMalloc(&g->rowc, sizeof(uint2) * (V + 1)));
-    CG(cudaMalloc(&g->arcs, sizeof(uint2) * std::max<i64>(A, 1)));
-    CG(cudaMalloc(&g->dist, sizeof(u32) * V));
-    CG(cudaMalloc(&g->xd, sizeof(u32) * (5 * V + 4)));  // sweep marks, two pull candidate lists, long scans
-    CG(cudaMalloc(&g->ctl, sizeof(Ctl)));
-    CG(cudaMalloc(&g->stats, sizeof(unsigned long long) * ST_N));
-    CG(cudaMalloc(&g->trace, sizeof(TraceEnt) * (TRACE_CAP + SAMPLE_CAP)));
+    CG(dalloc(&g->rowp, sizeof(longlong2) * (V + 1)));
+    CG(dalloc(&g->rowc, sizeof(uint2) * (V + 1)));
+    CG(dalloc(&g->arcs, sizeof(uint2) * std::max<i64>(A, 1)));
+    CG(dalloc(&g->dist, sizeof(u32) * V));
+    CG(dalloc(&g->xd, sizeof(u32) * (5 * V + 4)));  // sweep marks, two pull candidate lists, long scans
+    CG(dalloc(&g->ctl, sizeof(Ctl)));
+    CG(dalloc(&g->stats, sizeof(unsigned long long) * ST_N));
+    CG(dalloc(&g->trace, sizeof(TraceEnt) * (TRACE_CAP + SAMPLE_CAP)));
     CG(cudaMemsetAsync(g->ctl, 0, sizeof(Ctl), s));
     CG(cudaMemsetAsync(g->stats, 0, sizeof(unsigned long long) * ST_N, s));
     for (int i = 0; i < 4; ++i) CG(cudaEventCreate(&g->ev[i]));
-    CG(cudaMallocAsync(&d_row, sizeof(i64) * (V + 1), s));
-    CG(cudaMallocAsync(&d_flags, sizeof(u32) * 2, s));
+    CG(dalloc(&d_row, sizeof(i64) * (V + 1), s));
+    CG(dalloc(&d_flags, sizeof(u32) * 2, s));
     CG(cudaMemsetAsync(d_flags, 0, sizeof(u32) * 2, s));
     CG(cudaMemcpyAsync(d_row, row, sizeof(i64) * (V + 1), kind, s));
     if (A > 0) {
-      CG(cudaMallocAsync(&d_col, sizeof(u32) * A, s));
-      CG(cudaMallocAsync(&d_w, sizeof(u32) * A, s));
+      CG(dalloc(&d_col, sizeof(u32) * A, s));
+      CG(dalloc(&d_w, sizeof(u32) * A, s));
       CG(cudaMemcpyAsync(d_col, col, sizeof(u32) * A, kind, s));
       CG(cudaMemcpyAsync(d_w, weights, sizeof(u32) * A, kind, s));
     }
@@ -219,15 +286,15 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
     CG(cudaGetLastError());
     u32 flags[2] = {0, 0};
     CG(cudaMemcpyAsync(flags, d_flags, sizeof flags, cudaMemcpyDeviceToHost, s));
-    CG(cudaFreeAsync(d_row, s));
+    CG(cudaStreamSynchronize(s));  // the temporaries are free to go (plain or hooked frees)
+    CG(dfree(d_row, s));
     d_row = nullptr;
-    CG(cudaFreeAsync(d_flags, s));
+    CG(dfree(d_flags, s));
     d_flags = nullptr;
-    if (d_col) CG(cudaFreeAsync(d_col, s));
+    CG(dfree(d_col, s));
     d_col = nullptr;
-    if (d_w) CG(cudaFreeAsync(d_w, s));
+    CG(dfree(d_w, s));
     d_w = nullptr;
-    CG(cudaStreamSynchronize(s));
     if (flags[0]) {
       st = fail(SSSP_ERR_INVALID_ARGUMENT, "invalid CSR:%s%s%s%s", (flags[0] & 1) ? " row[0]!=0 or row[V]!=A" : "",
                 (flags[0] & 2) ? " row offsets decrease" : "", (flags[0] & 4) ? " col index >= V" : "",
@@ -238,10 +305,11 @@ extern "C" sssp_status sssp_graph_create(sssp_graph_t* out, int device, int64_t 
 #undef CG
   } while (0);
   if (st != SSSP_OK) {
-    if (d_row) cudaFree(d_row);
-    if (d_col) cudaFree(d_col);
-    if (d_w) cudaFree(d_w);
-    if (d_flags) cudaFree(d_flags);
+    cudaStreamSynchronize(g->stream);
+    dfree(d_row);
+    dfree(d_col);
+    dfree(d_w);
+    dfree(d_flags);
     return bail(st);
   }
   *out = g;
@@ -261,7 +329,7 @@ extern "C" void sssp_destroy(sssp_graph_t g) {
   void* ptrs[] = {g->rowp, g->rowc, g->arcs, g->old2new, g->new2old, g->dist, g->stage[0], g->stage[1], g->xd, g->ctl, g->sc,
                   g->items, g->hub_items, g->p2o, g->rowc_lv, g->ms_D, g->ms_Q, g->ms_items, g->ms_sc, g->ms_ctl, g->ms_stats, g->ms_src, g->stats, g->trace, g->out_tmp};
   for (void* p : ptrs)
-    if (p) cudaFree(p);
+    if (p) dfree(p);
   for (auto& e : g->ev)
     if (e) cudaEventDestroy(e);
   for (auto& e : g->ev_pool) cudaEventDestroy(e);
@@ -443,12 +511,12 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
   const u32 nh_cap = (u32)(A / EXPAND_HUB + 1);
   std::vector<void*> temps;
   auto alloc = [&](void** ptr, size_t bytes) -> cudaError_t {
-    cudaError_t e = cudaMalloc(ptr, std::max<size_t>(bytes, 4));
+    cudaError_t e = dalloc(ptr, std::max<size_t>(bytes, 4));
     if (e == cudaSuccess) temps.push_back(*ptr);
     return e;
   };
   auto free_all = [&]() {
-    for (void* t : temps) cudaFree(t);
+    for (void* t : temps) dfree(t);
     temps.clear();
   };
   u32 *hist = nullptr, *tmp = nullptr, *f[6] = {}, *dmax = nullptr, *key0 = nullptr, *key1 = nullptr,
@@ -463,8 +531,8 @@ extern "C" sssp_status sssp_reorder_ex(sssp_graph_t g, unsigned flags) {
     A_(alloc((void**)&tmp, sizeof(u32) * scan_tmp_elems(hist_n)));
     A_(alloc((void**)&dmax, sizeof(u32)));
     if (deg) {
-      if (!g->new2old) A_(cudaMalloc(&g->new2old, sizeof(u32) * V));
-      if (!g->old2new) A_(cudaMalloc(&g->old2new, sizeof(u32) * V));
+      if (!g->new2old) A_(dalloc(&g->new2old, sizeof(u32) * V));
+      if (!g->old2new) A_(dalloc(&g->old2new, sizeof(u32) * V));
       A_(alloc((void**)&key0, sizeof(u32) * V));
       A_(alloc((void**)&key1, sizeof(u32) * V));
       A_(alloc((void**)&id1, sizeof(u32) * V));
@@ -651,22 +719,23 @@ static sssp_status ensure_run_buffers(sssp_graph_t g, u32 K, u32 cap) {
   cudaStream_t s = g->stream;
   const u32 hub_cap = (u32)std::min<i64>(g->A / 2048 + 4096, 0x7FFFFFFF);
   if (K > g->K_alloc || cap != g->cap_alloc) {
-    if (g->items) CU(cudaFree(g->items));
-    if (g->sc) CU(cudaFree(g->sc));
-    if (g->p2o) CU(cudaFree(g->p2o));
+    if (g->items) CU(cudaStreamSynchronize(s));  // earlier runs may still read the old queues
+    if (g->items) CU(dfree(g->items));
+    if (g->sc) CU(dfree(g->sc));
+    if (g->p2o) CU(dfree(g->p2o));
     g->items = nullptr;
     g->sc = nullptr;
     g->p2o = nullptr;
-    CU(cudaMalloc(&g->items, sizeof(u64) * (size_t)K * cap));
-    CU(cudaMalloc(&g->p2o, sizeof(u32) * (((size_t)cap + 1) & ~(size_t)1) + sizeof(uint2) * (size_t)cap));
-    CU(cudaMalloc(&g->sc, sizeof(SlotCtl) * K));
+    CU(dalloc(&g->items, sizeof(u64) * (size_t)K * cap));
+    CU(dalloc(&g->p2o, sizeof(u32) * (((size_t)cap + 1) & ~(size_t)1) + sizeof(uint2) * (size_t)cap));
+    CU(dalloc(&g->sc, sizeof(SlotCtl) * K));
     CU(cudaMemsetAsync(g->sc, 0, sizeof(SlotCtl) * K, s));
     g->K_alloc = K;
     g->cap_alloc = cap;
     g->need_full_reset = true;
   }
   if (!g->hub_items) {
-    CU(cudaMalloc(&g->hub_items, sizeof(u64) * hub_cap));
+    CU(dalloc(&g->hub_items, sizeof(u64) * hub_cap));
     g->hub_cap = hub_cap;
     g->need_full_reset = true;
   }
@@ -740,7 +809,7 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   const bool adapt = dp.ai.mode != 0;
   if (adapt && pro && (!g->rowc_lv_valid || g->rowc_lv_g != dp.delta_bits)) {
     // heavy offsets for the light levels g << l (u32) / g * 2^l (f32), l = 0..4
-    if (!g->rowc_lv) CU(cudaMalloc(&g->rowc_lv, sizeof(uint2) * 5 * (size_t)(g->V + 1)));
+    if (!g->rowc_lv) CU(dalloc(&g->rowc_lv, sizeof(uint2) * 5 * (size_t)(g->V + 1)));
     for (u32 l = 0; l < 5; ++l) {
       const u32 th = f32 ? dp.delta_bits + (l << 23) : dp.delta_bits << l;
       k_heavy_offsets<<<grid_for(g->V), 256, 0, s>>>(g->rowp, g->arcs, g->V, th);
@@ -917,7 +986,7 @@ extern "C" sssp_status sssp_distances(sssp_graph_t g, void* out, sssp_memory whe
       dst = (u32*)pa.devicePointer;
     } else {
       cudaGetLastError();
-      if (!g->out_tmp) CU(cudaMalloc(&g->out_tmp, sizeof(u32) * g->V));
+      if (!g->out_tmp) CU(dalloc(&g->out_tmp, sizeof(u32) * g->V));
       staged = true;
     }
   }
@@ -953,7 +1022,7 @@ extern "C" sssp_status sssp_distances_async(sssp_graph_t g, void* out, sssp_memo
   }
   const int j = g->stage_next;
   g->stage_next ^= 1;
-  if (!g->stage[j]) CU(cudaMalloc(&g->stage[j], sizeof(u32) * g->V));
+  if (!g->stage[j]) CU(dalloc(&g->stage[j], sizeof(u32) * g->V));
   if (g->stage_used[j]) CU(cudaStreamWaitEvent(s, g->ev_out[j], 0));  // its previous copy is done
   // a8 into the staging buffer (HBM speed, run stream), then the copy engine moves it to
   // the host on d2h while the next sssp_run computes
@@ -1027,20 +1096,21 @@ extern "C" sssp_status sssp_run_multi(sssp_graph_t g, const int64_t* sources, in
   while (K < std::ceil(dp.ahead) + 2.0 && K < 64) K <<= 1;
   const u32 cap = (u32)std::min<i64>(g->V + g->V / 2 + g->A / 128 + 65536, 0x7FFFFFFF);
   if (!g->ms_D) {
-    CU(cudaMalloc(&g->ms_D, sizeof(u32) * MS_LANES * (size_t)g->V));
-    CU(cudaMalloc(&g->ms_Q, sizeof(u32) * (size_t)g->V));
-    CU(cudaMalloc(&g->ms_ctl, sizeof(MCtl)));
+    CU(dalloc(&g->ms_D, sizeof(u32) * MS_LANES * (size_t)g->V));
+    CU(dalloc(&g->ms_Q, sizeof(u32) * (size_t)g->V));
+    CU(dalloc(&g->ms_ctl, sizeof(MCtl)));
     CU(cudaMemsetAsync(g->ms_ctl, 0, sizeof(MCtl), s));
-    CU(cudaMalloc(&g->ms_stats, sizeof(unsigned long long) * MST_N));
-    CU(cudaMalloc(&g->ms_src, sizeof(u32) * 2 * MS_LANES));
+    CU(dalloc(&g->ms_stats, sizeof(unsigned long long) * MST_N));
+    CU(dalloc(&g->ms_src, sizeof(u32) * 2 * MS_LANES));
   }
   if (K > g->ms_K || cap > g->ms_cap) {
-    if (g->ms_items) CU(cudaFree(g->ms_items));
-    if (g->ms_sc) CU(cudaFree(g->ms_sc));
+    if (g->ms_items) CU(cudaStreamSynchronize(s));
+    if (g->ms_items) CU(dfree(g->ms_items));
+    if (g->ms_sc) CU(dfree(g->ms_sc));
     g->ms_items = nullptr;
     g->ms_sc = nullptr;
-    CU(cudaMalloc(&g->ms_items, sizeof(u64) * (size_t)K * cap));
-    CU(cudaMalloc(&g->ms_sc, sizeof(SlotCtl) * K));
+    CU(dalloc(&g->ms_items, sizeof(u64) * (size_t)K * cap));
+    CU(dalloc(&g->ms_sc, sizeof(SlotCtl) * K));
     CU(cudaMemsetAsync(g->ms_items, 0xFF, sizeof(u64) * (size_t)K * cap, s));
     CU(cudaMemsetAsync(g->ms_sc, 0, sizeof(SlotCtl) * K, s));
     g->ms_K = K;

@@ -882,3 +882,45 @@ def test_pull_symmetric_is_checked(sssp):
     with sssp.Graph(row, col, w) as G:
         G.reorder()
         assert G.is_symmetric()
+
+
+def test_allocator_hook_torch(sssp):
+    """sssp_set_allocator: with PyTorch's caching allocator behind the hook the
+    handle's buffers are torch allocations (memory_allocated grows by them and returns after
+    destroy), every hooked buffer is freed exactly once, and the SSSP is unchanged."""
+    import torch
+
+    g = gen.kronecker(12, 16, seed=21)
+    s = int(gen.sample_sources(g, 1, seed=2)[0])
+    exp = oracle.dijkstra(g.row, g.col, g.w, s)
+    log = {"alloc": 0, "free": 0, "live": {}}
+
+    def alloc(n, dev, stream):
+        p = torch.cuda.caching_allocator_alloc(n, dev, stream if stream else None)
+        log["alloc"] += 1
+        log["live"][p] = n
+        return p
+
+    def free(ptr, n, dev, stream):
+        assert log["live"].pop(ptr) == n
+        log["free"] += 1
+        torch.cuda.caching_allocator_delete(ptr)
+
+    torch.cuda.synchronize()
+    base = torch.cuda.memory_allocated()
+    sssp.sssp_set_allocator(alloc, free)
+    try:
+        with sssp.Graph(g.row, g.col, g.w) as G:
+            G.reorder()
+            G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+            assert_same(G.sssp(s, 16), exp, "torch allocator")
+            held = sum(log["live"].values())
+            assert log["alloc"] > 8 and held > 8 * g.A  # the arc array at least
+            assert torch.cuda.memory_allocated() - base >= held
+    finally:
+        sssp.sssp_set_allocator(None, None)
+    torch.cuda.synchronize()
+    assert log["free"] == log["alloc"] and not log["live"]
+    assert torch.cuda.memory_allocated() == base
+    with pytest.raises(sssp.SSSPError):  # one of the pair only
+        sssp._check(sssp._lib.sssp_set_allocator(sssp._ALLOC_FN(lambda *a: None), sssp._FREE_FN(), None), "x")
