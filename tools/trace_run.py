@@ -78,6 +78,26 @@ def main():
                       f"{sum(x['cyc_stage'] for x in xs)/n/1e3:6.2f} {sum(x['cyc_task'] for x in xs)/n/1e3:6.2f} "
                       f"{sum(x['cyc_tail'] for x in xs)/n/1e3:6.2f}   "
                       f"[{sum(x['tb_tasks'] for x in xs)/n/1e3:6.2f} {sum(x['ranges'] for x in xs)/n/1e3:6.2f}]")
+            # claim latency per sampled CTA: end of its previous batch -> end of this claim
+            # (diagnostics builds), with the unclaimed backlog (tail - claim position) it saw
+            per = collections.defaultdict(list)
+            for x in smp:
+                per[x["cta"]].append(x)
+            gaps = collections.defaultdict(list)
+            for xs in per.values():
+                xs.sort(key=lambda x: x["t_ns"])
+                for a_, b_ in zip(xs, xs[1:]):
+                    if a_.get("kind") == "batch" and b_.get("kind", "claim") == "claim" and b_["claimed"]:
+                        gaps[b_["cur"]].append(((b_["t_ns"] - a_["t_ns"]) / 1e3, b_["tail"] - b_["pos"], b_["claimed"]))
+            print("  claim latency (us, sampled CTAs: previous batch end -> claim end): bucket n  p50 p90 max"
+                  "  | backlog tail-pos at the claim p10 p50  | items p50")
+            for b in sorted(gaps):
+                g = sorted(x[0] for x in gaps[b])
+                bl = sorted(x[1] for x in gaps[b])
+                it = sorted(x[2] for x in gaps[b])
+                q = lambda v, f: v[min(len(v) - 1, int(f * len(v)))]
+                print(f"   bucket {b}: {len(g):5d}  {q(g,.5):7.2f} {q(g,.9):7.2f} {g[-1]:7.2f}  | {q(bl,.1):9d} {q(bl,.5):9d}"
+                      f"  | {q(it,.5):5d}")
             base = min((x["t_ns"] for x in smp), default=0)
             print(f"  samples: {len(smp)} (every 37th CTA's phase-1 claims); per bucket, 50 us windows: "
                   "t_us  claims  items  tail(max)  pend(max)")
