@@ -301,19 +301,27 @@ struct Smem {
 };
 
 // ---------------------------------------------------------------- helpers --
+#ifndef SSSP_LD_VOLATILE
+#define SSSP_LD_VOLATILE 0  // 0: probes and arc loads as plain asm (A/B: C4 -2 %, C3 -2 %, C1 -1 %)
+#endif
+#if SSSP_LD_VOLATILE
+#define SSSP_LD_ASM asm volatile
+#else
+#define SSSP_LD_ASM asm  // probes and arc loads are pure loads: let the compiler schedule them
+#endif
 // Filter probe of dist[] before the atomicMin (Alg. 1 l.2). Any value ever
 // stored in dist[v] is >= its current value, so a stale (L1-cached) read can
 // only cause an extra atomic, never a missed improvement.
 __device__ __forceinline__ u32 ld_probe(const u32* p, bool pred, u64 pol) {
   u32 v;
 #if SSSP_PROBE_L1
-  asm volatile(
+  SSSP_LD_ASM(
       "{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n mov.b32 %0, 0;\n"
       " @q ld.global.ca.L2::cache_hint.u32 %0, [%1], %3;\n}"
       : "=r"(v)
       : "l"(p), "r"((u32)pred), "l"(pol));
 #else
-  asm volatile(
+  SSSP_LD_ASM(
       "{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n mov.b32 %0, 0;\n"
       " @q ld.global.cg.L2::cache_hint.u32 %0, [%1], %3;\n}"
       : "=r"(v)
@@ -325,7 +333,7 @@ __device__ __forceinline__ u32 ld_probe(const u32* p, bool pred, u64 pol) {
 // Predicated arc load (streamed: L1 bypass, L2 evict-first). {0,0} if !pred.
 __device__ __forceinline__ uint2 ld_arc(const uint2* p, bool pred, u64 pol) {
   uint2 v;
-  asm volatile(
+  SSSP_LD_ASM(
       "{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n mov.b32 %0, 0;\n mov.b32 %1, 0;\n"
       " @q ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %4;\n}"
       : "=r"(v.x), "=r"(v.y)
