@@ -206,6 +206,7 @@ sssp_status sssp_export_csr(sssp_graph_t g, double delta, int64_t* rowlist, uint
 
 /* Tunables (defaults in brackets). Values are validated; takes effect at the
  * next sssp_run. */
+#define SSSP_BF_TAIL_DEFAULT 262144  /* entries: SSSP_PARAM_BF_TAIL's default */
 typedef enum {
     SSSP_PARAM_RING_SLOTS = 0,     /* K bucket queues, power of two in [4,64]; 0 = auto [0] */
     SSSP_PARAM_CTAS_PER_SM = 1,    /* persistent CTAs per SM; 0 = max co-resident [0] */
@@ -260,8 +261,20 @@ typedef enum {
                                       networks: thin frontiers; on dense ones the CTA-local
                                       depth-first order re-relaxes more). Same distances;
                                       0 = always through the global queue [1] */
-    SSSP_PARAM_LOCAL_LIMIT = 13    /* local-chase entries a CTA keeps (1..512); pushes beyond
+    SSSP_PARAM_LOCAL_LIMIT = 13,   /* local-chase entries a CTA keeps (1..512); pushes beyond
                                       go to the global queue, where idle CTAs can take them [512] */
+    SSSP_PARAM_BF_TAIL = 14        /* Bellman-Ford end: when a bucket closes, the ring's
+                                      queues hold at most this many entries, an earlier bucket
+                                      held at least 8x as many (the wave is past its peak) and
+                                      no push was dropped beyond the ring, the rest of the run is one
+                                      bucket [cur, inf): every queued vertex moves into it and
+                                      phase 1 relaxes all arcs (light and heavy) to quiescence.
+                                      Delta-stepping with Delta = inf is Bellman-Ford,
+                                      so the distances are the same; per-bucket statistics
+                                      (trace C_i, heavy relaxations) then stop at the switch.
+                                      Fixed Delta and the asynchronous phase 1 only; 0 = never;
+                                      -1 = auto: SSSP_BF_TAIL_DEFAULT on graphs with more than
+                                      8 arcs per vertex, never on sparser (road-like) ones [-1] */
 } sssp_param;
 sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t value);
 

@@ -51,6 +51,8 @@ SSSP_PARAM_MULTI_HUB_DELAY = 10
 SSSP_PARAM_PULL_SYMMETRIC = 11
 SSSP_PARAM_LOCAL_CHASE = 12
 SSSP_PARAM_LOCAL_LIMIT = 13
+SSSP_PARAM_BF_TAIL = 14
+SSSP_BF_TAIL_DEFAULT = 262144
 
 INF_U32 = 0xFFFFFFFF
 

@@ -164,17 +164,19 @@ struct __align__(128) Ctl {
   u32 lvl;           // light/heavy level of the current bucket: light iff w < g << lvl
   u32 csum;          // settled vertices of the current bucket (phase 2 / pull count them)
   u32 err_acc;       // OR of err over every run since the host last read it (k_seed keeps it)
-  u32 pad_a;
+  u32 bf;            // Bellman-Ford end: 0 off, 1 running (all arcs, one queue), 2 final clear
   // pull phases 2&3: candidate lists (unsettled vertices with arcs) in xd[V..3V); pull_sel = the
   // input list (2 = every vertex, the first pull), pull_n = list lengths
   u32 pull_sel, pull_n[2];
   u32 closed_c, closed_b;    // C_i and index of the bucket the last scheduler step closed (trace)
-  u32 pad_c;
+  u32 bf_t;          // switch to the Bellman-Ford end once the ring holds <= bf_t entries (0: never)
+  u32 bf_peak;       // most entries any closed bucket held (the end phase waits for the peak)
+  u32 pad_t;
   u64 t_first;               // earliest arrival at the current grid barrier (%globaltimer, trace)
   u32 long_n, long_head;     // pull: long scans handed to whole warps (count, claim tickets)
   u32 sample_n;              // phase-1 claim samples written (diagnostics)
   u32 first_n;               // the first pull's candidates: ids [0, first_n) (isolated ids excluded)
-  u32 pad_b[20];
+  u32 pad_b[18];
   u32 bar_count, pad3[31];   // own line: arrivals
   u32 bar_gen, pad4[31];     // own line: spun on
   u32 p2_head, pad5[31];     // own line: phase-2 static tickets
@@ -298,6 +300,7 @@ struct Smem {
   u32 mode, cur, lim, p2_begin, p2_end, sweep_first, round_end;
   u32 cur_end, rowc_off, theta_bits;  // bucket end (fine slots), light/heavy level
   u32 pull_sel, pull_n_in;            // pull phases 2&3: input candidate list
+  u32 bf;                             // Bellman-Ford end: phase 1 relaxes every arc
 };
 
 // ---------------------------------------------------------------- helpers --
@@ -745,13 +748,14 @@ __device__ __forceinline__ void process_batch(const Params& p, Smem& sm, const u
   // whole adjacency (predicate per arc). (Loading the rows with the dist probe, for stale
   // entries too, measured 4 % slower on C4.)
   const uint2* rowc = EXT ? p.rowc + sm.rowc_off : p.rowc;  // heavy offsets of the bucket's level
+  const bool bf_all = PH == 1 && sm.bf;  // Bellman-Ford end: phase 1 relaxes every arc
   auto range_of = [&](int i, i64& b, i64& e) {
     const u32 v = (u32)it[i] & ~CHUNK_FLAG;
     const uint2 r = rowc[v];
-    if (PRO && PH == 1) {
+    if (PRO && PH == 1 && !bf_all) {
       b = r.x;
       e = r.y;
-    } else {
+    } else {  // heavy range, the whole adjacency (no PRO) or, in the Bellman-Ford end, all arcs
       e = rowc[v + 1].x;
       b = (PRO && PH == 2) ? r.y : r.x;
     }
@@ -1152,9 +1156,9 @@ __device__ __forceinline__ uint4 ld_volatile_v4(const void* q) {
 __device__ bool decide_close_fast(const Params& p) {
   volatile Ctl* c = p.ctl;
   volatile SlotCtl* sc = p.sc;
-  u32 W[36];
+  u32 W[40];
 #pragma unroll
-  for (int i = 0; i < 9; ++i) {
+  for (int i = 0; i < 10; ++i) {
     const uint4 x = ld_volatile_v4(reinterpret_cast<const uint4*>(const_cast<Ctl*>(p.ctl)) + i);
     W[4 * i] = x.x;
     W[4 * i + 1] = x.y;
@@ -1164,9 +1168,12 @@ __device__ bool decide_close_fast(const Params& p) {
   static_assert(offsetof(Ctl, cur) == 0 && offsetof(Ctl, lim) == 4 && offsetof(Ctl, mode) == 8 &&
                 offsetof(Ctl, far_min) == 12 && offsetof(Ctl, p2_end) == 20 && offsetof(Ctl, epochs) == 28 &&
                 offsetof(Ctl, cur_end) == 64 && offsetof(Ctl, a_mode) == 68 && offsetof(Ctl, a_m) == 108 &&
-                offsetof(Ctl, csum) == 116 && offsetof(Ctl, pull_sel) == 128, "Ctl layout (decide_close_fast)");
+                offsetof(Ctl, csum) == 116 && offsetof(Ctl, bf) == 124 && offsetof(Ctl, pull_sel) == 128 &&
+                offsetof(Ctl, bf_t) == 148 && offsetof(Ctl, bf_peak) == 152 && offsetof(Ctl, bar_count) == 256,
+                "Ctl layout (decide_close_fast)");
   const u32 cur = W[0], lim0 = W[1], mode = W[2], fm = W[3], p2_end = W[5], epochs = W[7];
-  const u32 cur_end = W[16], a_mode = W[17], a_m = W[27], csum = W[29], pull_sel = W[32];
+  const u32 cur_end = W[16], a_mode = W[17], a_m = W[27], csum = W[29], pull_sel = W[32], bf_t = W[37];
+  const u32 bf_peak = W[38];
   if (a_mode) return false;
   const u32 s = cur & p.kmask;
   const u64 ws = sc[s].word;
@@ -1183,7 +1190,16 @@ __device__ bool decide_close_fast(const Params& p) {
       nxt_tail = t[k];
     }
   if (nxt == NONE && cur_end + 8 <= lim0 && cur_end + 8 > cur_end) return false;  // scan further: general path
+  const u32 peak = max(bf_peak, min((u32)(ws >> 32), p.cap));
+  if (bf_t && nxt != NONE && peak >= 8 * bf_t) {
+    // past the peak with few entries left: the general path decides on the Bellman-Ford end
+    u32 sum = 0;
+#pragma unroll
+    for (u32 k = 0; k < 8; ++k) sum += t[k];
+    if (sum <= bf_t) return false;
+  }
   sc[s].p2 = p2_end;
+  c->bf_peak = peak;
   if (mode == MODE_PULL || mode == MODE_PULL_LONG) c->pull_sel = pull_sel == 0 ? 1u : 0u;  // its output list
   c->csum = 0;
   c->closed_c = (p.claim_max & LOCAL_CHASE) ? NONE : csum;
@@ -1231,6 +1247,15 @@ __device__ void decide(const Params& p, u32 which) {
       return;
     }
     which = SYNC_P2;
+  }
+  if (which == SYNC_P1 && c->bf) {  // Bellman-Ford end quiescent: distances final
+    if (c->far_min != NONE) {  // a push was dropped (queue full): rebuild from dist[], go on
+      c->rescan_base = c->cur;
+    } else {
+      c->bf = 2;  // clear the queues (rescan_clear), then done
+    }
+    c->mode = MODE_RESCAN_CLEAR;
+    return;
   }
   if (which == SYNC_P1) {
     const u32 cur = c->cur, s = cur & p.kmask;
@@ -1322,6 +1347,39 @@ __device__ void decide(const Params& p, u32 which) {
     const u64 lim = (u64)nxt + K - 1;
     c->lim = (u32)min(lim, (u64)NONE - 1);
     c->cur = nxt;
+    c->bf_peak = max(c->bf_peak, t_items);
+    if (c->bf_t && !c->a_mode && !(p.flags & 2u) && fm == NONE && c->bf_peak >= 8 * c->bf_t) {
+      // Bellman-Ford end (Delta = inf for what is left): when the ring holds at most
+      // bf_t entries after the wave's peak (a closed bucket held >= 8 bf_t), the remaining buckets would each pay two grid barriers and a chain of
+      // round trips for a few thousand vertices. Instead every entry moves into bucket nxt's
+      // queue (MODE_MERGE), and one phase 1 relaxes all arcs (light and heavy) of every
+      // improved vertex until quiescence: a label-correcting fixpoint, so the same distances.
+      u32 tt[16], sum = 0, others = 0;
+#pragma unroll
+      for (u32 k = 0; k < 16; ++k)
+        tt[k] = (k < K && nxt + k <= c->lim) ? (u32)(sc[(nxt + k) & p.kmask].word >> 32) : 0u;
+#pragma unroll
+      for (u32 k = 0; k < 16; ++k) {
+        sum += tt[k];
+        others += k ? tt[k] : 0u;
+      }
+      bool more = false;  // a ring of more than 16 slots: the rest must be empty too
+      for (u32 k = 16; k < K && nxt + k <= c->lim; ++k) more |= (sc[(nxt + k) & p.kmask].word >> 32) != 0;
+      if (!more && sum <= c->bf_t) {
+        c->bf = 1;
+        c->epochs = c->epochs + 1;
+        if (others) {
+          c->cur_end = c->lim + 1;  // merge slots (nxt, lim] into slot nxt
+          c->mode = MODE_MERGE;
+        } else {
+          c->cur_end = NONE;
+          c->lim = NONE - 1;
+          c->round_end = min(tt[0], p.cap);
+          c->mode = MODE_PHASE1;
+        }
+        return;
+      }
+    }
     if (c->a_mode) adapt_next(p, t_items, c_i);
     c->cur_end = (u32)min((u64)nxt + c->a_m, (u64)c->lim + 1);
     c->epochs = c->epochs + 1;
@@ -1338,11 +1396,20 @@ __device__ void decide(const Params& p, u32 which) {
       sc[s].head = 0;
       sc[s].p2 = 0;
     }
+    if (c->bf == 2) {
+      c->bf = 0;
+      c->mode = MODE_DONE;
+      return;
+    }
     const u32 r = c->rescan_base;
     c->far_min = NONE;
     c->cur = r;
     c->lim = (u32)min((u64)r + K - 1, (u64)NONE - 1);
     c->cur_end = (u32)min((u64)r + c->a_m, (u64)c->lim + 1);
+    if (c->bf) {  // Bellman-Ford end: one bucket [r, inf)
+      c->lim = NONE - 1;
+      c->cur_end = NONE;
+    }
     c->mode = MODE_RESCAN_FILL;
   } else if (which == SYNC_MG) {  // slots (cur, cur_end) folded into slot cur
     for (u32 x = c->cur + 1; x < c->cur_end; ++x) {
@@ -1350,7 +1417,15 @@ __device__ void decide(const Params& p, u32 which) {
       sc[x & p.kmask].head = 0;
       sc[x & p.kmask].p2 = 0;
     }
-    if (c->far_min < c->cur_end) {  // slot cur overflowed while merging
+    if (c->bf) {  // merged for the Bellman-Ford end: one bucket [cur, inf)
+      c->cur_end = NONE;
+      c->lim = NONE - 1;
+      if (c->far_min != NONE) {  // slot cur overflowed while merging: rebuild from dist[]
+        c->rescan_base = c->cur;
+        c->mode = MODE_RESCAN_CLEAR;
+        return;
+      }
+    } else if (c->far_min < c->cur_end) {  // slot cur overflowed while merging
       enter_sweep(c);
       return;
     }
@@ -1386,6 +1461,8 @@ __device__ __forceinline__ void load_bucket(const Params& p, Smem& sm, volatile 
   const u32 l = vc->lvl;
   sm.rowc_off = (p.flags & 64u) ? l * (p.V + 1) : 0u;  // levels built only with PRO
   sm.theta_bits = l == 0 ? p.delta_bits : ((p.flags & 32u) ? p.delta_bits + (l << 23) : p.delta_bits << l);
+  sm.bf = vc->bf;
+  if (sm.bf) sm.theta_bits = NONE;  // without PRO: every arc counts as light
 }
 
 __device__ void grid_barrier(const Params& p, Smem& sm, u32 which) {
@@ -2144,10 +2221,14 @@ __device__ void pull_long(const Params& p, Smem& sm) {
 __device__ void rescan_clear(const Params& p) {
   const i64 t = (i64)blockIdx.x * blockDim.x + threadIdx.x;
   const i64 nt = (i64)gridDim.x * blockDim.x;
-  for (u32 s = 0; s < p.K; ++s) {
-    const u32 tail = min((u32)(ld_relaxed_u64(&p.sc[s].word) >> 32), p.cap);
-    u64* q = p.items + (u64)s * p.cap;
-    for (i64 i = t; i < tail; i += nt) st_relaxed_u64(q + i, SENTINEL);
+  for (u32 s0 = 0; s0 < p.K; s0 += 8) {
+    u32 tl[8];  // tails in flight together
+#pragma unroll
+    for (u32 k = 0; k < 8; ++k) tl[k] = s0 + k < p.K ? min((u32)(ld_relaxed_u64(&p.sc[s0 + k].word) >> 32), p.cap) : 0u;
+    for (u32 k = 0; k < 8 && s0 + k < p.K; ++k) {
+      u64* q = p.items + (u64)(s0 + k) * p.cap;
+      for (i64 i = t; i < tl[k]; i += nt) st_relaxed_u64(q + i, SENTINEL);
+    }
   }
 }
 
@@ -2220,18 +2301,32 @@ __device__ void merge_slots(const Params& p, Smem& sm) {
   u32 moved = 0;
   const i64 t0 = ((i64)blockIdx.x * blockDim.x + threadIdx.x) & ~31LL;
   const i64 nt = (i64)gridDim.x * blockDim.x;
-  for (u32 x = cur + 1; x < ce; ++x) {
-    const u32 sl = x & p.kmask;
-    const u32 tail = min((u32)(ld_relaxed_u64(&p.sc[sl].word) >> 32), p.cap);
-    u64* q = p.items + (u64)sl * p.cap;
-    for (i64 b = t0; b < tail; b += nt) {
+  for (u32 x0 = cur + 1; x0 < ce; x0 += 8) {
+    // eight slots at a time, their entries laid end to end: the tails in one round trip and
+    // every entry of the eight slots in one grid-stride pass (the Bellman-Ford end merges a
+    // few thousand entries spread over up to K - 1 slots)
+    u32 tl[8], tot = 0;
+#pragma unroll
+    for (u32 k = 0; k < 8; ++k)
+      tl[k] = x0 + k < ce ? min((u32)(ld_relaxed_u64(&p.sc[(x0 + k) & p.kmask].word) >> 32), p.cap) : 0u;
+#pragma unroll
+    for (u32 k = 0; k < 8; ++k) tot += tl[k];
+    for (i64 b = t0; b < tot; b += nt) {
       const i64 i = b + lane;
       bool want[UNROLL] = {};
       u32 vv[UNROLL] = {}, dd[UNROLL] = {};
-      if (i < tail) {
-        const u64 e = ld_relaxed_u64(q + i);
-        st_relaxed_u64(q + i, SENTINEL);
-        if (e != SENTINEL) {
+      if (i < tot) {
+        u32 k = 0, o = (u32)i;
+#pragma unroll
+        for (u32 j = 0; j < 7; ++j)
+          if (k == j && o >= tl[j]) {
+            o -= tl[j];
+            k = j + 1;
+          }
+        u64* q = p.items + (u64)((x0 + k) & p.kmask) * p.cap + o;
+        const u64 e = ld_relaxed_u64(q);
+        st_relaxed_u64(q, SENTINEL);
+        if (e != SENTINEL && !((u32)e & CHUNK_FLAG)) {
           vv[0] = (u32)e;
           dd[0] = (u32)(e >> 32);
           want[0] = ld_cg(p.dist + vv[0]) == dd[0];
@@ -2294,8 +2389,8 @@ __global__ void __launch_bounds__(DS_THREADS, SSSP_MINB) k_delta_step(Params p) 
     } else if (mode == MODE_PULL_LONG) {
       pull_long<F32, PRO>(p, sm);
       grid_barrier(p, sm, SYNC_P2);
-    } else if (ABL && mode == MODE_MERGE) {  // extended build only (adaptive Delta)
-      if constexpr (ABL) merge_slots<F32>(p, sm);
+    } else if (mode == MODE_MERGE) {  // adaptive Delta (extended build) / Bellman-Ford end
+      merge_slots<F32>(p, sm);
       grid_barrier(p, sm, SYNC_MG);
     } else if (ABL && mode == MODE_P2_COMPACT) {  // extended build only (edge-balanced phase 2)
       if constexpr (ABL) p2_compact<F32, PRO>(p, sm);
@@ -2345,6 +2440,7 @@ struct AdaptInit {
   float d0;        // Delta_0 in fine units
   u32 m0, mmin, mmax, lvl0;
   u32 first_n;     // ids [0, first_n) hold every vertex with arcs and the source
+  u32 bf_t;        // Bellman-Ford end threshold (entries left in the ring; 0 = never)
 };
 __global__ void k_seed(Params p, u32 src, AdaptInit ai) {
   const u32 t = threadIdx.x;
@@ -2398,6 +2494,9 @@ __global__ void k_seed(Params p, u32 src, AdaptInit ai) {
     c->long_n = c->long_head = 0;
     c->sample_n = 0;
     c->first_n = ai.first_n;
+    c->bf = 0;
+    c->bf_t = ai.bf_t;
+    c->bf_peak = 0;
   }
 }
 

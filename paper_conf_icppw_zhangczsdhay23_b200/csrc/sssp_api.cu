@@ -171,7 +171,7 @@ struct sssp_graph_s {
   int64_t kt_launches = 0;
   bool run_timed = false, reorder_timed = false;
   // params
-  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP;
+  i64 p_ring = 0, p_ctas = 0, p_cap = 0, p_claim = BATCH, p_l2 = 1, p_adwl = 1, p_sync = 0, p_p2eb = -1, p_adapt = 0, p_align = 1, p_hub_delay = 0, p_pull = 0, p_local = 1, p_local_lim = LOC_CAP, p_bf = -1;
   i64 hub_ids_cached = -1;
   int sym_state = -1;  // arc multiset symmetric? -1 unknown (checked on demand after a weight sort)
   i64 v_nz = -1;       // degree-sorted graphs: vertices with arcs are ids [0, v_nz); -1 unknown
@@ -422,6 +422,10 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
     case SSSP_PARAM_LOCAL_CHASE:
       if (v < 0 || v > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "local chase is 0, 1 or 2");
       g->p_local = v;
+      return SSSP_OK;
+    case SSSP_PARAM_BF_TAIL:
+      if (v < -1 || v > 0x7FFFFFFF) return fail(SSSP_ERR_INVALID_ARGUMENT, "Bellman-Ford end threshold -1 (auto) or in [0, 2^31)");
+      g->p_bf = v;
       return SSSP_OK;
     case SSSP_PARAM_LOCAL_LIMIT:
       if (v < 1 || v > (i64)LOC_CAP) return fail(SSSP_ERR_INVALID_ARGUMENT, "local limit in [1,%u]", LOC_CAP);
@@ -881,6 +885,11 @@ static sssp_status launch_run(sssp_graph_t g, u32 src_internal, const DeltaParam
   }
   AdaptInit ai = dp.ai;
   ai.first_n = (g->pro_flags & SSSP_PRO_DEGREE) ? (u32)std::max<i64>(g->v_nz, (i64)src_internal + 1) : (u32)g->V;
+  // fixed Delta, asynchronous phase 1 only; auto (-1): on dense graphs (A > 8 V). On sparse,
+  // road-like ones the remaining vertices form long chains that label-correcting re-relaxes
+  // (C2: 6 % slower with it).
+  const i64 bf = g->p_bf >= 0 ? g->p_bf : (g->A > 8 * g->V ? (i64)SSSP_BF_TAIL_DEFAULT : 0);
+  ai.bf_t = (ai.mode != 0 || g->p_sync) ? 0u : (u32)bf;
   // a5: init (Alg. 2 l.1-3)
   k_fill_u32<<<grid_for(g->V), 256, 0, s>>>(g->dist, g->V, f32 ? 0x7F800000u : 0xFFFFFFFFu);
   k_seed<<<1, 64, 0, s>>>(p, src_internal, ai);

@@ -118,6 +118,7 @@ def test_grid_many_buckets(sssp):
         with sssp.Graph(g.row, g.col, g.w) as G:
             if reorder:
                 G.reorder()
+            G.set_param(sssp.SSSP_PARAM_BF_TAIL, 0)  # every bucket on its own
             for d in (50, 400, 1600):
                 assert_same(G.sssp(s, d), exp, f"grid reorder={reorder} delta={d}")
                 st = G.stats()
@@ -286,6 +287,7 @@ def test_stats_invariants(sssp):
         with sssp.Graph(g.row, g.col, g.w) as G:
             G.reorder()
             G.set_param(sssp.SSSP_PARAM_P2_EDGE_BALANCED, eb)
+            G.set_param(sssp.SSSP_PARAM_BF_TAIL, 0)  # per-bucket heavy relaxations to the end
             G.sssp(s, 32)
             st = G.stats()
         _check_stats(st, reach, heavy_deg, reach_new)
@@ -495,6 +497,7 @@ def test_bucket_settled_counts_match_oracle(sssp, case):
         if case != "kron-noreorder":
             G.reorder()
         G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1 if case == "kron-pull" else 0)
+        G.set_param(sssp.SSSP_PARAM_BF_TAIL, 0)  # every bucket closed on its own
         if case == "grid":  # with the local chase on (auto here) the counts are not kept
             G.sssp(srcs[0], 1600)
             assert all(e["closed_c"] == INF for e in G.trace() if e["closed_b"] != INF)
@@ -924,3 +927,47 @@ def test_allocator_hook_torch(sssp):
     assert torch.cuda.memory_allocated() == base
     with pytest.raises(sssp.SSSPError):  # one of the pair only
         sssp._check(sssp._lib.sssp_set_allocator(sssp._ALLOC_FN(lambda *a: None), sssp._FREE_FN(), None), "x")
+
+
+# ------------------------------------------------- Bellman-Ford end ----
+@pytest.mark.parametrize("case", ["kron-pull", "kron-push", "kron-noreorder", "grid", "kron-f32"])
+def test_bf_tail_parity(sssp, case):
+    """SSSP_PARAM_BF_TAIL: once the ring holds <= threshold entries, the rest of the run is
+    one bucket [cur, inf) relaxing every arc (Delta = inf is Bellman-Ford).
+    Bit-exact with the oracle for thresholds 0 (never), small (the last buckets), the
+    default, and 2^30 (never reached: the wave's peak must hold 8x the threshold), with the
+    merge of non-empty ring slots, and with a tiny queue capacity (dropped pushes -> rescans);
+    the end phase must actually run in the small-threshold case (fewer buckets)."""
+    if case == "grid":
+        g, deltas = gen.grid(200, 150, p=0.2, seed=9), (50, 400)
+    elif case == "kron-f32":
+        g, deltas = gen.kronecker(13, 16, seed=77, weights="f32"), (0.02, 0.1)
+    else:
+        g, deltas = gen.kronecker(13, 16, seed=76), (4, 16, 64)
+    srcs = [int(x) for x in gen.sample_sources(g, 2, seed=11)]
+    exp = {s: oracle.dijkstra(g.row, g.col, g.w, s) for s in srcs}
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        if case != "kron-noreorder":
+            G.reorder()
+        if case in ("kron-pull", "kron-f32"):
+            G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        if case == "grid":  # the CTA-local chase keeps the buckets' queues short: no peak to pass
+            for s in srcs:
+                G.set_param(sssp.SSSP_PARAM_BF_TAIL, 256)
+                assert_same(G.sssp(s, deltas[0]), exp[s], f"grid local chase bf_tail=256 src={s}")
+            G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, 0)
+        nb = {}
+        for t in (0, 64, 256, -1, sssp.SSSP_BF_TAIL_DEFAULT, 1 << 30):
+            G.set_param(sssp.SSSP_PARAM_BF_TAIL, t)
+            for d in deltas:
+                for s in srcs:
+                    assert_same(G.sssp(s, d), exp[s], f"{case} bf_tail={t} delta={d} src={s}")
+                    nb[(t, d, s)] = G.stats()["buckets"]
+        ran = sum(nb[(256, d, s)] < nb[(0, d, s)] for d in deltas for s in srcs)
+        assert ran > 0, f"{case}: the Bellman-Ford end never ran at threshold 256"
+        G.set_param(sssp.SSSP_PARAM_SLOT_CAPACITY, 4096)  # pushes dropped: rescans inside the end phase
+        G.set_param(sssp.SSSP_PARAM_BF_TAIL, 256)
+        for s in srcs:
+            assert_same(G.sssp(s, deltas[0]), exp[s], f"{case} bf_tail=256 capacity=4096 src={s}")
+        with pytest.raises(sssp.SSSPError):
+            G.set_param(sssp.SSSP_PARAM_BF_TAIL, -2)
