@@ -258,6 +258,11 @@ def main():
 
         torch.cuda.set_device(dev)
         if backend == "nccl":
+            # communicator setup lines (nranks, NVLS / P2P transport) on stderr, so the one JSON
+            # line stays alone on stdout and the driver can check the communicator size
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
         else:
             dist.init_process_group(backend)
