@@ -57,6 +57,21 @@ def main():
                 G.set_param(sssp.SSSP_PARAM_LOCAL_CHASE, local)
                 same(G.sssp(s, d), exp, f"local chase {local} V={g.V}")
     print("sanitize cases local chase: OK", flush=True)
+    # Bellman-Ford end (SSSP_PARAM_BF_TAIL): the merge of non-empty ring slots, the all-arc phase 1,
+    # the final clear, and the rescan inside the end phase (tiny queue capacity); pull phases on
+    g = gen.kronecker(11, 16, seed=76)
+    srcs = [int(x) for x in gen.sample_sources(g, 2, seed=11)]
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.set_param(sssp.SSSP_PARAM_CTAS_PER_SM, 1)
+        G.reorder()
+        G.set_param(sssp.SSSP_PARAM_PULL_SYMMETRIC, 1)
+        for t, cap in ((16, 0), (64, 0), (64, 4096)):
+            G.set_param(sssp.SSSP_PARAM_BF_TAIL, t)
+            G.set_param(sssp.SSSP_PARAM_SLOT_CAPACITY, cap)
+            for s in srcs:
+                for d in (4, 16):
+                    same(G.sssp(s, d), oracle.dijkstra(g.row, g.col, g.w, s), f"bf_tail={t} cap={cap} d={d}")
+    print("sanitize cases Bellman-Ford end: OK", flush=True)
 
 
 if __name__ == "__main__":
