@@ -440,6 +440,11 @@ extern "C" sssp_status sssp_set_param(sssp_graph_t g, sssp_param p, int64_t v) {
 }
 
 // ------------------------------------------------------------- symmetry --
+template <int NF>
+static sssp_status radix_pass(sssp_graph_t g, Fields<NF>& a, Fields<NF>& b, int kf, i64 n, int sh,
+                              u32* hist, u32* tmp);
+static int bits_for(u64 maxv);
+
 extern "C" sssp_status sssp_is_symmetric(sssp_graph_t g, int* out) {
   NvtxRange nvtx_("sssp_is_symmetric");
   sssp_status st = check_handle(g);
@@ -454,7 +459,34 @@ extern "C" sssp_status sssp_is_symmetric(sssp_graph_t g, int* out) {
     u32 h = 0;
     CU(cudaMallocAsync(&flag, sizeof(u32), s));
     CU(cudaMemsetAsync(flag, 0, sizeof(u32), s));
-    if (g->A > 0) {
+    const int vb = std::max(1, bits_for((u64)(g->V - 1))), wb = bits_for(g->maxw_bits);
+    bool sorted_done = false;
+    if (g->A > 0 && 2 * vb + wb <= 64) {
+      // sort-based: transposed keys, the PRO radix passes, one compare (falls back to the
+      // per-run binary searches below if the temporaries do not fit)
+      const i64 A = g->A, ntiles = (A + RS_TILE - 1) / RS_TILE;
+      u32 *f[4] = {}, *hist = nullptr, *tmp = nullptr;
+      bool ok = true;
+      for (int i = 0; i < 4 && ok; ++i) ok = dalloc(&f[i], sizeof(u32) * A) == cudaSuccess;
+      ok = ok && dalloc(&hist, sizeof(u32) * 256 * ntiles) == cudaSuccess;
+      ok = ok && dalloc(&tmp, sizeof(u32) * scan_tmp_elems(256 * ntiles)) == cudaSuccess;
+      if (ok) {
+        const SymPack pk{vb, wb};
+        const unsigned nbv = (unsigned)std::min<i64>((g->V + 7) / 8, (i64)g->num_sms * 64);
+        k_sym_keys<<<nbv, 256, 0, s>>>(g->rowp, g->arcs, g->V, pk, f[0], f[1]);
+        Fields<2> a{{f[0], f[1]}}, b{{f[2], f[3]}};
+        for (int sh = 0; sh < 2 * vb + wb && !st; sh += 8) st = radix_pass<2>(g, a, b, sh >= 32 ? 1 : 0, A, sh & 31, hist, tmp);
+        if (!st) k_sym_compare<<<nbv, 256, 0, s>>>(g->rowp, g->arcs, g->V, pk, a.f[0], a.f[1], flag);
+        CU(cudaGetLastError());
+        cudaStreamSynchronize(s);  // before the temporaries are freed
+        sorted_done = !st;
+      }
+      cudaGetLastError();
+      for (u32* x : {f[0], f[1], f[2], f[3], hist, tmp})
+        if (x) dfree(x);
+      if (st) return st;
+    }
+    if (g->A > 0 && !sorted_done) {
       const i64 nb = std::min<i64>((g->A + SYM_PER_BLOCK - 1) / SYM_PER_BLOCK, (i64)g->num_sms * 16);
       k_check_symmetric<<<(unsigned)nb, 256, 0, s>>>(g->rowp, g->arcs, g->V, g->A, flag);
       CU(cudaGetLastError());

@@ -971,3 +971,31 @@ def test_bf_tail_parity(sssp, case):
             assert_same(G.sssp(s, deltas[0]), exp[s], f"{case} bf_tail=256 capacity=4096 src={s}")
         with pytest.raises(sssp.SSSPError):
             G.set_param(sssp.SSSP_PARAM_BF_TAIL, -2)
+
+
+@pytest.mark.parametrize("wt,scale", [("u32", 12), ("f32", 12), ("f32", 17)])
+def test_symmetry_check_paths(sssp, wt, scale):
+    """sssp_is_symmetric has two exact paths: the sort-based one (transposed keys radix-sorted
+    and compared with the arcs, when (dst, w, src) packs into 64 bits: u32 s12, f32 s12) and the
+    per-run binary searches (f32 s17: 17 + 32 + 17 bits do not pack). Both must accept the
+    symmetrised graph and reject it after one arc's weight changes by one ulp/unit."""
+    g = gen.kronecker(scale, 8, seed=91, weights=wt)
+    with sssp.Graph(g.row, g.col, g.w) as G:
+        G.reorder()
+        assert G.is_symmetric()
+    w = g.w.copy()
+    k = len(w) // 3
+    w[k] = np.nextafter(w[k], np.float32(np.inf)) if wt == "f32" else w[k] + 1
+    with sssp.Graph(g.row, g.col, w) as G:
+        G.reorder()
+        assert not G.is_symmetric()
+    # a self-loop-free directed copy: drop one arc of a symmetric pair
+    keep = np.ones(len(g.col), bool)
+    keep[k] = False
+    u = np.repeat(np.arange(g.V), np.diff(g.row))[keep]
+    row = np.zeros(g.V + 1, np.int64)
+    np.add.at(row, u + 1, 1)
+    row = np.cumsum(row)
+    with sssp.Graph(row, g.col[keep].copy(), g.w[keep].copy()) as G:
+        G.reorder()
+        assert not G.is_symmetric()
